@@ -1,0 +1,313 @@
+#!/usr/bin/env python
+"""Benchmark: batched dgbtrf + dgbtrs (the whole hot path) on B200.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config C3] [--impl ours|reference]
+
+One STEP = dgbtrf_strided_batched + dgbtrs_strided_batched (two launches of
+our sm_100a kernels through the C ABI) over one batch of synthetic band
+matrices resident in HBM.  Default workload: BASELINE.json's target config
+"batch=10000, n=512, kl=ku=10, nrhs=1 ... at 1/2/4/8 B200" (C3).  Multi-GPU:
+one process per GPU (torchrun), each rank factors its own contiguous shard
+(10000 matrices per GPU, weak scaling), no collective on the data path; the
+time is the max over ranks.  Before every step the pristine A/B are restored
+by a device-to-device copy OUTSIDE the timed events; A (1.27 GB per GPU at
+C3) is ~10x the 126 MB L2, so inputs are larger than L2.
+
+Reported: value = effective GFLOP/s (nominal, pivot-independent flop count of
+SURVEY 8(d)); hbm_gbs = algorithmic bytes (exact SURVEY 8(d) forms) / time;
+roofline for the dominant kernel vs MEASURED_PEAKS.json hbm_gbs; e2e through
+the host-buffer C-ABI entry point (H2D + D2H inside the timed region);
+cpu_baseline = the CPU oracle (test infrastructure) timed on a bounded sample
+on the host cores.  --impl reference runs that oracle as the reference arm.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "batched dgbtrf+dgbtrs Gflop/s & HBM GB/s (% roofline) vs n,kl,ku at 1/2/4/8 B200"
+CONFIGS = {  # name: (batch per GPU, n, kl, ku, nrhs, description)
+    "C1": (100, 64, 2, 2, 1, "configs[0]: batch=100, n=64, kl=ku=2, nrhs=1"),
+    "C2": (10000, 256, 1, 1, 1, "configs[1]: tridiagonal-like batch=10000, n=256, kl=ku=1, nrhs=1"),
+    "C3": (10000, 512, 10, 10, 1, "configs[2]: batch=10000/GPU, n=512, kl=ku=10, nrhs=1 (north_star target)"),
+    "C4": (5000, 1024, 2, 32, 16, "configs[3]: batch=5000, n=1024, kl=2, ku=32, nrhs=16"),
+}
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d.get("hbm_gbs", 6650.0)), "measured"
+    return 6650.0, "fallback"
+
+
+def ncu_traffic(kernel: str, cfg: str):
+    """dram bytes per launch for `kernel` at `cfg` from the committed ncu summary, else None."""
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        d = json.load(open(p))
+        e = d[cfg][kernel]
+        return float(e["dram_bytes_read"]) + float(e["dram_bytes_write"])
+    except Exception:
+        return None
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.idx = gpu_index
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.idx), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "50"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"], "samples": 0}
+        time.sleep(0.12)
+        self.proc.terminate()
+        try:
+            out, _ = self.proc.communicate(timeout=5)
+        except Exception:
+            self.proc.kill()
+            out = ""
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in out.strip().splitlines():
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 6:
+                continue
+            try:
+                sm.append(float(f[0])); smax.append(float(f[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[2:6]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def cpu_oracle_rate(n, kl, ku, nrhs, seconds=6.0, sample=None):
+    """The CPU oracle (OpenMP over the batch, all host threads) on a bounded
+    sample of the workload; returns (matrices/s, sample size, threads, reps)."""
+    import oracle
+    from paper_conf_sc_abdelfattahtlad23_b200 import inputs as I
+    if sample is None:
+        sample = 1024
+    A0 = I.gen_band(n, n, kl, ku, count=sample)
+    B0 = I.gen_rhs(n, nrhs, count=sample)
+    oracle.build()
+    threads = oracle.max_threads()
+    best = None
+    reps = 0
+    t_end = time.perf_counter() + seconds
+    while reps < 3 or time.perf_counter() < t_end:
+        A, B = A0.copy(), B0.copy()
+        t0 = time.perf_counter()
+        ipiv, info = oracle.dgbtrf(A, n, n, kl, ku)
+        oracle.dgbtrs(A, ipiv, B, n, kl, ku)
+        dt = time.perf_counter() - t0
+        best = dt if best is None else min(best, dt)
+        reps += 1
+        if reps >= 50:
+            break
+    return sample / best, sample, threads, reps
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=100)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", default="C3", choices=sorted(CONFIGS))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    bpg, n, kl, ku, nrhs, desc = CONFIGS[args.config]
+    from paper_conf_sc_abdelfattahtlad23_b200 import inputs as I
+    b_trf, b_trs = I.alg_bytes(n, n, kl, ku, nrhs)
+    f_trf, f_trs = I.nominal_flops(n, kl, ku, nrhs)
+    config = {"workload": desc, "batch_per_gpu": bpg, "global_batch": bpg * world, "n": n, "kl": kl, "ku": ku,
+              "nrhs": nrhs, "ldab": 2 * kl + ku + 1, "layout": "strided LAPACK band", "parallelism": f"batch-shard x{world}",
+              "l2": "inputs larger than L2" if bpg * n * (2 * kl + ku + 1) * 8 > 2 * 126e6
+              else "L2 flushed (256 MB write) before every timed step"}
+
+    if args.impl == "reference":
+        # Reference arm for this tier = the CPU oracle, rank 0 only.
+        if rank != 0:
+            return
+        rate, sample, threads, reps = cpu_oracle_rate(n, kl, ku, nrhs, seconds=max(3.0, 0.5 * args.steps))
+        gflops = rate * (f_trf + f_trs) / 1e9
+        line = {"impl": "reference", "metric": METRIC, "value": gflops, "unit": "GFLOP/s", "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * bpg * world / rate,
+                "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+                "data": "synthetic (seeded counter-based U(-1,1) bands)", "config": config,
+                "matrices_per_s": rate,
+                "cpu_baseline": {"value": gflops, "unit": "GFLOP/s", "cores": threads, "kind": "oracle",
+                                 "sample": f"{sample} matrices of the workload, best of {reps} runs"},
+                "e2e": {"value": gflops, "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+        print(json.dumps(line))
+        return
+
+    import torch
+    import torch.distributed as dist
+    import paper_conf_sc_abdelfattahtlad23_b200 as bl
+
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    dev = torch.device("cuda", torch.cuda.current_device())
+    bl.load()
+
+    # ---- inputs: this rank's shard of the global batch (counter-based generator)
+    lo, hi = I.shard_range(bpg * world, rank, world)
+    cnt = hi - lo
+    A0 = torch.from_numpy(I.gen_band(n, n, kl, ku, count=cnt, first=lo)).to(dev)
+    B0 = torch.from_numpy(I.gen_rhs(n, nrhs, count=cnt, first=lo)).to(dev)
+    A = torch.empty_like(A0)
+    B = torch.empty_like(B0)
+    P = torch.zeros((cnt, n), dtype=torch.int32, device=dev)
+    info = torch.zeros(cnt, dtype=torch.int32, device=dev)
+    flush = None if config["l2"].startswith("inputs larger") else torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    st = torch.cuda.current_stream()
+
+    def step(evs=None):
+        A.copy_(A0)
+        B.copy_(B0)
+        if flush is not None:
+            flush.zero_()
+        if evs is not None:
+            evs[0].record(st)
+        bl.dgbtrf_strided_batched(n, n, kl, ku, A, P, info)
+        if evs is not None:
+            evs[1].record(st)
+        bl.dgbtrs_strided_batched("N", n, kl, ku, A, P, B)
+        if evs is not None:
+            evs[2].record(st)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    assert int(info.abs().sum()) == 0
+
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.steps)]
+    sampler = ClockSampler(torch.cuda.current_device()) if rank == 0 else None
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    if sampler:
+        sampler.start()
+    for k in range(args.steps):
+        step(evs[k])
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clocks = sampler.stop() if sampler else None
+    t_trf = [e[0].elapsed_time(e[1]) for e in evs]
+    t_trs = [e[1].elapsed_time(e[2]) for e in evs]
+    tot_ms = sum(a + b for a, b in zip(t_trf, t_trs))
+    tl = torch.tensor([tot_ms, sum(t_trf), sum(t_trs)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(tl, op=dist.ReduceOp.MAX)
+    tot_ms, trf_ms, trs_ms = tl.tolist()
+    ms_step = tot_ms / args.steps
+    glob = bpg * world
+    value = glob * (f_trf + f_trs) / (ms_step * 1e-3) / 1e9
+    hbm = glob * (b_trf + b_trs) / (ms_step * 1e-3) / 1e9
+
+    # ---- e2e through the host-buffer C-ABI entry point (H2D + D2H timed)
+    Ah = torch.from_numpy(I.gen_band(n, n, kl, ku, count=cnt, first=lo)).pin_memory()
+    Bh = torch.from_numpy(I.gen_rhs(n, nrhs, count=cnt, first=lo)).pin_memory()
+    Ahw, Bhw = torch.empty_like(Ah).pin_memory(), torch.empty_like(Bh).pin_memory()
+    Ph = torch.zeros((cnt, n), dtype=torch.int32).pin_memory()
+    Ih = torch.zeros(cnt, dtype=torch.int32).pin_memory()
+    e2e_ms = []
+    for k in range(args.e2e_steps + 1):
+        Ahw.copy_(Ah); Bhw.copy_(Bh)
+        if world > 1:
+            dist.barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(st)
+        bl.dgbsv_strided_batched_host(n, kl, ku, Ahw, Ph, Bhw, Ih)  # synchronous
+        e1.record(st)
+        torch.cuda.synchronize()
+        if k > 0:
+            e2e_ms.append(e0.elapsed_time(e1))
+    te = torch.tensor([sum(e2e_ms) / len(e2e_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+    e2e_step = te.item()
+    h2d = Ah.numel() * 8 + Bh.numel() * 8
+    d2h = Ah.numel() * 8 + Ph.numel() * 4 + Bh.numel() * 8 + Ih.numel() * 4
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    peak, peak_kind = peaks()
+    dom = "gbtrf_window_kernel" if trf_ms >= trs_ms else "gbtrs_window_kernel"
+    dom_ms = (trf_ms if trf_ms >= trs_ms else trs_ms) / args.steps
+    dom_bytes = cnt * (b_trf if trf_ms >= trs_ms else b_trs)
+    achieved = dom_bytes / (dom_ms * 1e-3) / 1e9
+    traffic = ncu_traffic(dom, args.config)
+    line = {
+        "metric": METRIC, "value": value, "unit": "GFLOP/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded counter-based U(-1,1) bands, NaN fill/corners)",
+        "config": config,
+        "hbm_gbs": hbm, "hbm_frac_of_8TBs": hbm / 8000.0, "hbm_frac_of_measured": hbm / peak,
+        "matrices_per_s": glob / (ms_step * 1e-3),
+        "kernels": {"gbtrf_ms": trf_ms / args.steps, "gbtrs_ms": trs_ms / args.steps,
+                    "gbtrf_gbs": cnt * b_trf / (trf_ms / args.steps * 1e-3) / 1e9,
+                    "gbtrs_gbs": cnt * b_trs / (trs_ms / args.steps * 1e-3) / 1e9,
+                    "variant_trf": bl.trf_variant(n, n, kl, ku), "variant_trs": bl.trs_variant(n, kl, ku, nrhs)},
+        "roofline": {"kernel": dom, "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "peak_kind": peak_kind, "traffic": traffic,
+                     "alg_bytes_per_launch": dom_bytes},
+        "e2e": {"value": glob * (f_trf + f_trs) / (e2e_step * 1e-3) / 1e9, "unit": "GFLOP/s",
+                "ms_per_step": e2e_step, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+                "api": "dgbsv_strided_batched_host (pinned host buffers)"},
+        "gpu_launches": 2 * args.steps,
+        "clocks": clocks,
+    }
+    if world == 1 and not args.no_cpu:
+        rate, sample, threads, reps = cpu_oracle_rate(n, kl, ku, nrhs)
+        line["cpu_baseline"] = {"value": rate * (f_trf + f_trs) / 1e9, "unit": "GFLOP/s", "cores": threads,
+                                "kind": "oracle", "matrices_per_s": rate,
+                                "sample": f"{sample} matrices of the workload, best of {reps} runs"}
+    print(json.dumps(line))
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,155 @@
+/*
+ * bandlu.h -- C ABI of the B200-native batched band LU / solve library.
+ *
+ * Operations (PAPER.md = Abdelfattah et al., SC-W 2023, text at
+ * /root/reference/PAPER.md; "P:<line>"):
+ *   dgbtrf : LU factorization with partial pivoting of a batch of m x n band
+ *            matrices, kl sub- / ku super-diagonals (Sec. 5, P:336-567;
+ *            interface P:314-318; column algorithm).
+ *   dgbtrs : solve A X = B with the factors (Sec. 6; interface
+ *            P:320-326), TRANS = 'N'.
+ *   dgbsv  : dgbtrf then dgbtrs (Sec. 3, Sec. 7 P:686-702;
+ *            interface P:328-333).
+ * Semantics are LAPACK DGBTRF(DGBTF2)/DGBTRS/DGBSV, which the paper adopts
+ * (P:26-27): results equal the reference CPU oracle (oracle/) --
+ * pivots and info bit-exact; factors and solutions bitwise in practice
+ * (same fp64 operation sequence), criterion 1e-12 relative entrywise.
+ *
+ * ---------------------------------------------------------------- layout
+ * A (band storage, LAPACK, P:286-304 and Fig. 2): each matrix is a
+ *   column-major array AB(ldab, n), ldab >= 2*kl+ku+1.  With kv = kl+ku and
+ *   0-based indices, A(i,j) is stored at AB[j*ldab + kv+i-j].  Rows 0..kl-1
+ *   are fill-in space: their input values are never read.  On exit rows
+ *   0..kv hold U (upper bandwidth kv) and rows kv+1..2kl+ku hold the
+ *   multipliers of L (not permuted by later interchanges, "swap to the right
+ *   only").  Positions whose matrix row is outside [0, m) ("corners")
+ *   and padding rows ldab > 2kl+ku+1 are never read and never written, except
+ *   that -- exactly as LAPACK DGBTF2's fill-in zeroing does -- fill-row
+ *   positions of columns < n whose matrix row is >= m are set to 0 when m < n.
+ * ipiv: min(m,n) int32 per matrix, 1-based LAPACK convention:
+ *   row j was interchanged with row ipiv[j]-1, ipiv[j] in [j+1, min(m,j+1+kl)].
+ * info: one int32 per matrix ("dedicated return code in the info
+ *   array"): 0 = success, k > 0 = U(k,k) (1-based) is exactly zero; the
+ *   factorization is still completed.  Written for every matrix when
+ *   batch > 0, also on the quick return m = 0 or n = 0.
+ * B: each right-hand side block is column-major B(ldb, nrhs), ldb >= max(1,n);
+ *   rows n..ldb-1 are untouched.
+ *
+ * ------------------------------------------------------- memory / calls
+ * All array arguments are DEVICE pointers (pointer-array variants: a device
+ * array of device pointers) unless the name ends in _host.  Calls
+ * are asynchronous on `stream` (a cudaStream_t; NULL = legacy default
+ * stream); results are valid after the stream is synchronized.  The caller
+ * owns all memory; the device entry points keep no state and allocate
+ * nothing.  Thread-safe, re-entrant, deterministic (no atomics in the
+ * arithmetic); per-matrix results do not depend on batch, its sharding, or
+ * the kernel variant chosen.
+ * Strided variants: matrix b starts at dA + b*strideA (strideA >= ldab*n),
+ * dipiv + b*strideP (strideP >= min(m,n)), dB + b*strideB (strideB >=
+ * ldb*nrhs); overlapping matrices are undefined behaviour.
+ *
+ * ------------------------------------------------------------- errors
+ * Return 0: work enqueued.  Return -k: argument k (1-based position in the
+ * C signature) is illegal; LAPACK numbering is kept where LAPACK has the
+ * argument (trf: -1 m, -2 n, -3 kl, -4 ku, -6 ldab; trs: -1 trans, -2 n,
+ * -3 kl, -4 ku, -5 nrhs, -7 ldab, -10 ldb; gbsv: -1 n, -2 kl, -3 ku,
+ * -4 nrhs, -6 ldab, -9 ldb); batch < 0, a NULL array with batch > 0, or a
+ * too-small stride return the position of that argument.  Nothing is
+ * enqueued when the return is nonzero.  BANDLU_ERR_UNSUPPORTED: trans other
+ * than 'N'/'n' (transposed solve not implemented yet).  BANDLU_ERR_CUDA +
+ * (cudaError_t) : a launch/runtime error (enqueue failed).
+ */
+#ifndef BANDLU_H
+#define BANDLU_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* binary compatible with cudaStream_t */
+typedef struct CUstream_st *bandlu_stream_t;
+
+#define BANDLU_ERR_UNSUPPORTED 1000
+#define BANDLU_ERR_CUDA 2000
+
+/* Kernel variant selector for the *_ex entry points (testing / profiling).
+ * AUTO = the library heuristic (what the plain entry points use). */
+enum bandlu_variant {
+    BANDLU_AUTO = 0,
+    BANDLU_GENERIC = 1, /* warp-per-matrix in-place kernel, any m, n, kl, ku (safeguard) */
+    BANDLU_WINDOW = 2   /* register-resident sliding window, compiled (kl, ku) only (Sec. 5.3 / 8.1) */
+};
+
+/* ---- dgbtrf: band LU with partial pivoting ---- */
+int dgbtrf_batched(int m, int n, int kl, int ku,
+                   double *const *dA_array, int ldab,
+                   int *const *dipiv_array, int *dinfo,
+                   int batch, bandlu_stream_t stream);
+int dgbtrf_strided_batched(int m, int n, int kl, int ku,
+                           double *dA, int ldab, int64_t strideA,
+                           int *dipiv, int64_t strideP, int *dinfo,
+                           int batch, bandlu_stream_t stream);
+
+/* ---- dgbtrs: A X = B with the dgbtrf factors, trans = 'N'.
+ * LAPACK DGBTRS semantics: no singularity check (singular U gives Inf/NaN). */
+int dgbtrs_batched(char trans, int n, int kl, int ku, int nrhs,
+                   const double *const *dA_array, int ldab,
+                   const int *const *dipiv_array,
+                   double *const *dB_array, int ldb,
+                   int batch, bandlu_stream_t stream);
+int dgbtrs_strided_batched(char trans, int n, int kl, int ku, int nrhs,
+                           const double *dA, int ldab, int64_t strideA,
+                           const int *dipiv, int64_t strideP,
+                           double *dB, int ldb, int64_t strideB,
+                           int batch, bandlu_stream_t stream);
+
+/* ---- dgbsv: dgbtrf + dgbtrs.  B is untouched for every matrix
+ * with info > 0 (LAPACK DGBSV). ---- */
+int dgbsv_batched(int n, int kl, int ku, int nrhs,
+                  double *const *dA_array, int ldab, int *const *dipiv_array,
+                  double *const *dB_array, int ldb, int *dinfo,
+                  int batch, bandlu_stream_t stream);
+int dgbsv_strided_batched(int n, int kl, int ku, int nrhs,
+                          double *dA, int ldab, int64_t strideA,
+                          int *dipiv, int64_t strideP,
+                          double *dB, int ldb, int64_t strideB, int *dinfo,
+                          int batch, bandlu_stream_t stream);
+
+/* ---- host-buffer end-to-end variant of dgbsv_strided_batched: hA, hipiv,
+ * hB, hinfo are HOST pointers (pinned memory recommended).  The library
+ * allocates device memory from the stream-ordered pool, copies A and B in,
+ * factors and solves, copies A (factors), ipiv, B (solution) and info back,
+ * and synchronizes `stream` before returning.  Work is pipelined over batch
+ * chunks so copies overlap the kernels.  Returns as above, or
+ * BANDLU_ERR_CUDA + err on an allocation / copy failure. */
+int dgbsv_strided_batched_host(int n, int kl, int ku, int nrhs,
+                               double *hA, int ldab, int64_t strideA,
+                               int *hipiv, int64_t strideP,
+                               double *hB, int ldb, int64_t strideB, int *hinfo,
+                               int batch, bandlu_stream_t stream);
+
+/* ---- variant-forcing entry points (tests / profiling).  variant is an
+ * enum bandlu_variant; forcing BANDLU_WINDOW for a (kl, ku) that is not
+ * compiled returns BANDLU_ERR_UNSUPPORTED. ---- */
+int dgbtrf_strided_batched_ex(int m, int n, int kl, int ku,
+                              double *dA, int ldab, int64_t strideA,
+                              int *dipiv, int64_t strideP, int *dinfo,
+                              int batch, bandlu_stream_t stream, int variant);
+int dgbtrs_strided_batched_ex(char trans, int n, int kl, int ku, int nrhs,
+                              const double *dA, int ldab, int64_t strideA,
+                              const int *dipiv, int64_t strideP,
+                              double *dB, int ldb, int64_t strideB,
+                              int batch, bandlu_stream_t stream, int variant);
+
+/* Which variant AUTO picks for a shape (no launch). */
+int bandlu_trf_variant(int m, int n, int kl, int ku);
+int bandlu_trs_variant(int n, int kl, int ku, int nrhs);
+/* Number of kernels one call enqueues for a shape (accounting for bench). */
+int bandlu_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* BANDLU_H */

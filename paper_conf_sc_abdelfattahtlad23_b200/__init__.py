@@ -1,0 +1,14 @@
+"""B200-native batched band LU with partial pivoting (dgbtrf) and banded
+solve (dgbtrs / dgbsv), after Abdelfattah et al., SC-W 2023.
+
+The product is libbandlu.so (C ABI, include/bandlu.h; sm_100a CUDA kernels in
+csrc/).  ``binding`` marshals torch CUDA tensors into it; ``inputs`` is the
+seeded synthetic workload generator.  Nothing here imports oracle/.
+"""
+from .binding import (AUTO, GENERIC, WINDOW, BandLUError, dgbsv_batched, dgbsv_strided_batched,  # noqa: F401
+                      dgbsv_strided_batched_host, dgbtrf_batched, dgbtrf_strided_batched, dgbtrs_batched,
+                      dgbtrs_strided_batched, load, ptr_array, trf_variant, trs_variant)
+
+__all__ = ["dgbtrf_strided_batched", "dgbtrs_strided_batched", "dgbsv_strided_batched", "dgbtrf_batched",
+           "dgbtrs_batched", "dgbsv_batched", "dgbsv_strided_batched_host", "ptr_array", "load",
+           "trf_variant", "trs_variant", "AUTO", "GENERIC", "WINDOW", "BandLUError"]

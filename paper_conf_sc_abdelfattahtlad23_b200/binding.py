@@ -1,0 +1,190 @@
+"""Thin ctypes binding over the C ABI in include/bandlu.h (argument
+marshalling only -- every step of the hot path runs in libbandlu.so's sm_100a
+kernels).  There is no CPU fallback: if the shared library is missing or a
+call fails, a RuntimeError is raised.
+
+Tensor conventions (SURVEY 8(b) "Python view"): a strided batch of band
+matrices is a contiguous float64 CUDA tensor A[batch, n, ldab] (column-major
+AB(ldab, n) per matrix), ipiv int32 [batch, min(m, n)], info int32 [batch],
+B float64 [batch, nrhs, ldb].  Calls are enqueued on torch's current CUDA
+stream (or `stream=`), asynchronously.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import torch
+
+from . import _build
+
+AUTO, GENERIC, WINDOW = 0, 1, 2
+ERR_UNSUPPORTED, ERR_CUDA = 1000, 2000
+
+_lib = None
+
+
+class BandLUError(RuntimeError):
+    def __init__(self, fn: str, code: int):
+        if code < 0:
+            msg = f"{fn}: argument {-code} is illegal"
+        elif code == ERR_UNSUPPORTED:
+            msg = f"{fn}: unsupported (variant / trans)"
+        elif code >= ERR_CUDA:
+            msg = f"{fn}: CUDA error {code - ERR_CUDA}"
+        else:
+            msg = f"{fn}: error {code}"
+        super().__init__(msg)
+        self.code = code
+
+
+def lib_path() -> str:
+    return _build.LIB
+
+
+def load(build_if_missing: bool = False):
+    """Load libbandlu.so (raise if it is missing: no fallback path exists)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(_build.LIB):
+        if build_if_missing:
+            _build.build()
+        else:
+            raise RuntimeError(f"CUDA extension {_build.LIB} not built; run __graft_entry__.build()")
+    lib = ctypes.CDLL(_build.LIB)
+    i, i64, p, ch = ctypes.c_int, ctypes.c_int64, ctypes.c_void_p, ctypes.c_char
+    sig = {
+        "dgbtrf_batched": [i, i, i, i, p, i, p, p, i, p],
+        "dgbtrf_strided_batched": [i, i, i, i, p, i, i64, p, i64, p, i, p],
+        "dgbtrf_strided_batched_ex": [i, i, i, i, p, i, i64, p, i64, p, i, p, i],
+        "dgbtrs_batched": [ch, i, i, i, i, p, i, p, p, i, i, p],
+        "dgbtrs_strided_batched": [ch, i, i, i, i, p, i, i64, p, i64, p, i, i64, i, p],
+        "dgbtrs_strided_batched_ex": [ch, i, i, i, i, p, i, i64, p, i64, p, i, i64, i, p, i],
+        "dgbsv_batched": [i, i, i, i, p, i, p, p, i, p, i, p],
+        "dgbsv_strided_batched": [i, i, i, i, p, i, i64, p, i64, p, i, i64, p, i, p],
+        "dgbsv_strided_batched_host": [i, i, i, i, p, i, i64, p, i64, p, i, i64, p, i, p],
+        "bandlu_trf_variant": [i, i, i, i],
+        "bandlu_trs_variant": [i, i, i, i],
+        "bandlu_version": [],
+    }
+    for name, args in sig.items():
+        f = getattr(lib, name)
+        f.argtypes = args
+        f.restype = ctypes.c_int
+    _lib = lib
+    return lib
+
+
+# exported symbol list (checked by tests against include/bandlu.h)
+EXPORTS = ("dgbtrf_batched", "dgbtrf_strided_batched", "dgbtrf_strided_batched_ex", "dgbtrs_batched",
+           "dgbtrs_strided_batched", "dgbtrs_strided_batched_ex", "dgbsv_batched", "dgbsv_strided_batched",
+           "dgbsv_strided_batched_host", "bandlu_trf_variant", "bandlu_trs_variant", "bandlu_version")
+
+
+def _stream(stream):
+    if stream is None:
+        return ctypes.c_void_p(torch.cuda.current_stream().cuda_stream)
+    if isinstance(stream, torch.cuda.Stream):
+        return ctypes.c_void_p(stream.cuda_stream)
+    return ctypes.c_void_p(int(stream))
+
+
+def _ptr(t: torch.Tensor | None):
+    return ctypes.c_void_p(t.data_ptr() if t is not None and t.numel() > 0 else 0)
+
+
+def _chk(fn: str, code: int):
+    if code != 0:
+        raise BandLUError(fn, code)
+
+
+def _dev(t: torch.Tensor, dtype, name: str, ndim: int):
+    if not (t.is_cuda and t.dtype == dtype and t.dim() == ndim and t.is_contiguous()):
+        raise TypeError(f"{name}: need a contiguous CUDA {dtype} tensor of rank {ndim}")
+
+
+def dgbtrf_strided_batched(m: int, n: int, kl: int, ku: int, A: torch.Tensor, ipiv: torch.Tensor,
+                           info: torch.Tensor, variant: int = AUTO, stream=None) -> None:
+    """In place: A [batch, n, ldab] -> LU factors; ipiv [batch, >=min(m,n)]; info [batch]."""
+    _dev(A, torch.float64, "A", 3); _dev(ipiv, torch.int32, "ipiv", 2); _dev(info, torch.int32, "info", 1)
+    batch, n_, ldab = A.shape
+    if n_ != n:
+        raise ValueError("A.shape[1] must be n")
+    f = load().dgbtrf_strided_batched_ex
+    _chk("dgbtrf_strided_batched", f(m, n, kl, ku, _ptr(A), ldab, n * ldab, _ptr(ipiv), ipiv.shape[1],
+                                     _ptr(info), batch, _stream(stream), variant))
+
+
+def dgbtrs_strided_batched(trans: str, n: int, kl: int, ku: int, A: torch.Tensor, ipiv: torch.Tensor,
+                           B: torch.Tensor, variant: int = AUTO, stream=None) -> None:
+    """In place: B [batch, nrhs, ldb] <- A^{-1} B using dgbtrf factors."""
+    _dev(A, torch.float64, "A", 3); _dev(ipiv, torch.int32, "ipiv", 2); _dev(B, torch.float64, "B", 3)
+    batch, _, ldab = A.shape
+    _, nrhs, ldb = B.shape
+    f = load().dgbtrs_strided_batched_ex
+    _chk("dgbtrs_strided_batched", f(trans.encode()[:1], n, kl, ku, nrhs, _ptr(A), ldab, n * ldab, _ptr(ipiv),
+                                     ipiv.shape[1], _ptr(B), ldb, nrhs * ldb, batch, _stream(stream), variant))
+
+
+def dgbsv_strided_batched(n: int, kl: int, ku: int, A: torch.Tensor, ipiv: torch.Tensor, B: torch.Tensor,
+                          info: torch.Tensor, stream=None) -> None:
+    _dev(A, torch.float64, "A", 3); _dev(ipiv, torch.int32, "ipiv", 2); _dev(B, torch.float64, "B", 3)
+    _dev(info, torch.int32, "info", 1)
+    batch, _, ldab = A.shape
+    _, nrhs, ldb = B.shape
+    _chk("dgbsv_strided_batched", load().dgbsv_strided_batched(
+        n, kl, ku, nrhs, _ptr(A), ldab, n * ldab, _ptr(ipiv), ipiv.shape[1], _ptr(B), ldb, nrhs * ldb,
+        _ptr(info), batch, _stream(stream)))
+
+
+def ptr_array(ts) -> torch.Tensor:
+    """Device array of device pointers for the pointer-array entry points."""
+    ptrs = [t.data_ptr() for t in ts]
+    dev = ts[0].device if len(ts) else torch.device("cuda")
+    return torch.tensor(ptrs, dtype=torch.int64, device=dev)
+
+
+def dgbtrf_batched(m: int, n: int, kl: int, ku: int, A_ptrs: torch.Tensor, ldab: int, ipiv_ptrs: torch.Tensor,
+                   info: torch.Tensor, batch: int, stream=None) -> None:
+    _chk("dgbtrf_batched", load().dgbtrf_batched(m, n, kl, ku, _ptr(A_ptrs), ldab, _ptr(ipiv_ptrs), _ptr(info),
+                                                 batch, _stream(stream)))
+
+
+def dgbtrs_batched(trans: str, n: int, kl: int, ku: int, nrhs: int, A_ptrs: torch.Tensor, ldab: int,
+                   ipiv_ptrs: torch.Tensor, B_ptrs: torch.Tensor, ldb: int, batch: int, stream=None) -> None:
+    _chk("dgbtrs_batched", load().dgbtrs_batched(trans.encode()[:1], n, kl, ku, nrhs, _ptr(A_ptrs), ldab,
+                                                 _ptr(ipiv_ptrs), _ptr(B_ptrs), ldb, batch, _stream(stream)))
+
+
+def dgbsv_batched(n: int, kl: int, ku: int, nrhs: int, A_ptrs: torch.Tensor, ldab: int, ipiv_ptrs: torch.Tensor,
+                  B_ptrs: torch.Tensor, ldb: int, info: torch.Tensor, batch: int, stream=None) -> None:
+    _chk("dgbsv_batched", load().dgbsv_batched(n, kl, ku, nrhs, _ptr(A_ptrs), ldab, _ptr(ipiv_ptrs), _ptr(B_ptrs),
+                                               ldb, _ptr(info), batch, _stream(stream)))
+
+
+def dgbsv_strided_batched_host(n: int, kl: int, ku: int, A: torch.Tensor, ipiv: torch.Tensor, B: torch.Tensor,
+                               info: torch.Tensor, stream=None) -> None:
+    """End-to-end: HOST tensors (pinned recommended) in and out; synchronous."""
+    for t, d, nm in ((A, torch.float64, "A"), (ipiv, torch.int32, "ipiv"), (B, torch.float64, "B"),
+                     (info, torch.int32, "info")):
+        if t.is_cuda or t.dtype != d or not t.is_contiguous():
+            raise TypeError(f"{nm}: need a contiguous host {d} tensor")
+    batch, _, ldab = A.shape
+    _, nrhs, ldb = B.shape
+    _chk("dgbsv_strided_batched_host", load().dgbsv_strided_batched_host(
+        n, kl, ku, nrhs, _ptr(A), ldab, n * ldab, _ptr(ipiv), ipiv.shape[1], _ptr(B), ldb, nrhs * ldb,
+        _ptr(info), batch, _stream(stream)))
+
+
+def raw_call(name: str, *args) -> int:
+    """Call an ABI entry point with raw ctypes arguments; returns its code (tests)."""
+    return getattr(load(), name)(*args)
+
+
+def trf_variant(m: int, n: int, kl: int, ku: int) -> int:
+    return load().bandlu_trf_variant(m, n, kl, ku)
+
+
+def trs_variant(n: int, kl: int, ku: int, nrhs: int) -> int:
+    return load().bandlu_trs_variant(n, kl, ku, nrhs)

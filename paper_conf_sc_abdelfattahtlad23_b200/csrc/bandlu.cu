@@ -1,0 +1,403 @@
+// bandlu.cu -- C ABI host layer (include/bandlu.h): argument checking with
+// LAPACK error numbering, quick returns, kernel-variant dispatch (the B200
+// counterpart of the paper's "complete picture", Sec. 5.4
+// P:558-567, and its tuning sweep P:526-556), launches.  No allocation and no
+// host synchronisation on the device entry points.
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <cstdio>
+#include <mutex>
+
+#include "../../include/bandlu.h"
+#include "common.cuh"
+#include "gbtrf_window.cuh"
+#include "gbtrs_window.cuh"
+#include "generic.cuh"
+
+using namespace bandlu;
+
+namespace {
+
+// (KL, KU) pairs compiled into register-resident window kernels (PAPER.md
+// Sec. 8.1 P:897-929 proposes per-(kl, ku) specialisation; we instantiate the
+// bands of the paper's sweeps and of BASELINE.json's configs).
+#define BANDLU_WINDOW_LIST(X) \
+    X(0, 0)                   \
+    X(0, 3)                   \
+    X(1, 1)                   \
+    X(2, 2)                   \
+    X(2, 3)                   \
+    X(3, 0)                   \
+    X(3, 2)                   \
+    X(4, 4)                   \
+    X(10, 7)                  \
+    X(10, 10)                 \
+    X(2, 32)
+
+inline int cuda_ret(cudaError_t e) { return e == cudaSuccess ? 0 : BANDLU_ERR_CUDA + (int)e; }
+
+template <class K>
+int set_smem(K kernel, size_t bytes) {
+    if (bytes > 48 * 1024) {
+        cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+        if (e != cudaSuccess) return cuda_ret(e);
+    }
+    return 0;
+}
+
+// ------------------------------------------------------------------ trf
+template <int KL, int KU, class AP, class PP>
+int launch_trf_window(int m, int n, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st) {
+    using C = TrfWin<KL, KU>;
+    auto k = gbtrf_window_kernel<KL, KU, AP, PP>;
+    size_t sm = C::smem_bytes();
+    if (int r = set_smem(k, sm)) return r;
+    const int64_t per_block = (int64_t)C::WARPS * C::GPW;
+    const unsigned grid = (unsigned)((batch + per_block - 1) / per_block);
+    k<<<grid, C::WARPS * 32, sm, st>>>(m, n, A, ldab, P, info, batch);
+    return cuda_ret(cudaGetLastError());
+}
+
+template <class AP, class PP>
+int launch_trf_generic(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st) {
+    const unsigned grid = (unsigned)(((int64_t)batch * 32 + 127) / 128);
+    gbtrf_generic_kernel<AP, PP><<<grid, 128, 0, st>>>(m, n, kl, ku, A, ldab, P, info, batch);
+    return cuda_ret(cudaGetLastError());
+}
+
+bool trf_window_available(int kl, int ku) {
+#define X(a, b) \
+    if (kl == a && ku == b) return true;
+    BANDLU_WINDOW_LIST(X)
+#undef X
+    return false;
+}
+
+int pick_trf(int m, int n, int kl, int ku) {
+    if (m <= 0 || n <= 0) return BANDLU_GENERIC;
+    return trf_window_available(kl, ku) ? BANDLU_WINDOW : BANDLU_GENERIC;
+}
+
+template <class AP, class PP>
+int run_trf(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st, int variant) {
+    if (batch == 0) return 0;
+    if (variant == BANDLU_AUTO) variant = pick_trf(m, n, kl, ku);
+    if (variant == BANDLU_WINDOW && m > 0 && n > 0) {
+#define X(a, b) \
+    if (kl == a && ku == b) return launch_trf_window<a, b>(m, n, A, ldab, P, info, batch, st);
+        BANDLU_WINDOW_LIST(X)
+#undef X
+        return BANDLU_ERR_UNSUPPORTED;
+    }
+    if (variant != BANDLU_GENERIC && variant != BANDLU_WINDOW) return BANDLU_ERR_UNSUPPORTED;
+    return launch_trf_generic(m, n, kl, ku, A, ldab, P, info, batch, st);
+}
+
+// ------------------------------------------------------------------ trs
+template <int KL, int KU, class AP, class PP, class BP>
+int launch_trs_window(int n, int nrhs, AP A, int ldab, PP P, BP B, int ldb, const int *skip, int batch,
+                      cudaStream_t st) {
+    using C = TrsWin<KL, KU>;
+    const int R = nrhs >= 32 ? 32 : pow2_ceil(nrhs);
+    const int chunks = (nrhs + 31) / 32;
+    auto k = gbtrs_window_kernel<KL, KU, AP, PP, BP>;
+    const size_t sm = C::smem_bytes(R);
+    if (int r = set_smem(k, sm)) return r;
+    const int64_t units = (int64_t)batch * chunks;
+    const int gpw = 32 / R;
+    const unsigned grid = (unsigned)((units + gpw - 1) / gpw);
+    k<<<grid, 32, sm, st>>>(n, nrhs, A, ldab, P, B, ldb, skip, batch, R, chunks);
+    return cuda_ret(cudaGetLastError());
+}
+
+template <class AP, class PP, class BP>
+int launch_trs_generic(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ldb, const int *skip,
+                       int batch, cudaStream_t st) {
+    const int64_t threads = (int64_t)batch * nrhs;
+    const unsigned grid = (unsigned)((threads + 127) / 128);
+    gbtrs_generic_kernel<AP, PP, BP><<<grid, 128, 0, st>>>(n, kl, ku, nrhs, A, ldab, P, B, ldb, skip, batch);
+    return cuda_ret(cudaGetLastError());
+}
+
+int pick_trs(int n, int kl, int ku, int nrhs) {
+    (void)n;
+    (void)nrhs;
+    return trf_window_available(kl, ku) ? BANDLU_WINDOW : BANDLU_GENERIC;
+}
+
+template <class AP, class PP, class BP>
+int run_trs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ldb, const int *skip, int batch,
+            cudaStream_t st, int variant) {
+    if (batch == 0 || n == 0 || nrhs == 0) return 0;
+    if (variant == BANDLU_AUTO) variant = pick_trs(n, kl, ku, nrhs);
+    if (variant == BANDLU_WINDOW) {
+#define X(a, b) \
+    if (kl == a && ku == b) return launch_trs_window<a, b>(n, nrhs, A, ldab, P, B, ldb, skip, batch, st);
+        BANDLU_WINDOW_LIST(X)
+#undef X
+        return BANDLU_ERR_UNSUPPORTED;
+    }
+    if (variant != BANDLU_GENERIC) return BANDLU_ERR_UNSUPPORTED;
+    return launch_trs_generic(n, kl, ku, nrhs, A, ldab, P, B, ldb, skip, batch, st);
+}
+
+// ------------------------------------------------------------ arg checks
+int check_trf(int m, int n, int kl, int ku, const void *A, int ldab, int64_t strideA, const void *P,
+              int64_t strideP, const void *info, int batch, bool strided) {
+    if (m < 0) return -1;
+    if (n < 0) return -2;
+    if (kl < 0) return -3;
+    if (ku < 0) return -4;
+    if (ldab < 2 * kl + ku + 1) return -6;
+    if (strided) {  // (m,n,kl,ku,dA,ldab,strideA,dipiv,strideP,dinfo,batch)
+        if (batch < 0) return -11;
+        if (batch > 0) {
+            if (!A) return -5;
+            if (strideA < (int64_t)ldab * n) return -7;
+            if (!P && m > 0 && n > 0) return -8;
+            if (strideP < (int64_t)(m < n ? m : n)) return -9;
+            if (!info) return -10;
+        }
+    } else {  // (m,n,kl,ku,dA_array,ldab,dipiv_array,dinfo,batch)
+        if (batch < 0) return -9;
+        if (batch > 0) {
+            if (!A) return -5;
+            if (!P && m > 0 && n > 0) return -7;
+            if (!info) return -8;
+        }
+    }
+    return 0;
+}
+
+int check_trs(char trans, int n, int kl, int ku, int nrhs, const void *A, int ldab, int64_t strideA, const void *P,
+              int64_t strideP, const void *B, int ldb, int64_t strideB, int batch, bool strided) {
+    if (trans != 'N' && trans != 'n' && trans != 'T' && trans != 't' && trans != 'C' && trans != 'c') return -1;
+    if (n < 0) return -2;
+    if (kl < 0) return -3;
+    if (ku < 0) return -4;
+    if (nrhs < 0) return -5;
+    if (ldab < 2 * kl + ku + 1) return -7;
+    if (strided) {  // (trans,n,kl,ku,nrhs,dA,ldab,strideA,dipiv,strideP,dB,ldb,strideB,batch)
+        if (ldb < (n > 1 ? n : 1)) return -12;
+        if (batch < 0) return -14;
+        if (batch > 0 && n > 0 && nrhs > 0) {
+            if (!A) return -6;
+            if (strideA < (int64_t)ldab * n) return -8;
+            if (!P) return -9;
+            if (strideP < n) return -10;
+            if (!B) return -11;
+            if (strideB < (int64_t)ldb * nrhs) return -13;
+        }
+    } else {
+        if (ldb < (n > 1 ? n : 1)) return -10;  // (trans,n,kl,ku,nrhs,dA_array,ldab,dipiv_array,dB_array,ldb,batch)
+        if (batch < 0) return -11;
+        if (batch > 0 && n > 0 && nrhs > 0) {
+            if (!A) return -6;
+            if (!P) return -8;
+            if (!B) return -9;
+        }
+    }
+    if (trans != 'N' && trans != 'n') return BANDLU_ERR_UNSUPPORTED;
+    return 0;
+}
+
+}  // namespace
+
+// =================================================================== ABI
+extern "C" {
+
+int bandlu_version(void) { return 1; }
+
+int bandlu_trf_variant(int m, int n, int kl, int ku) { return pick_trf(m, n, kl, ku); }
+int bandlu_trs_variant(int n, int kl, int ku, int nrhs) { return pick_trs(n, kl, ku, nrhs); }
+
+int dgbtrf_strided_batched_ex(int m, int n, int kl, int ku, double *dA, int ldab, int64_t strideA, int *dipiv,
+                              int64_t strideP, int *dinfo, int batch, bandlu_stream_t stream, int variant) {
+    if (int r = check_trf(m, n, kl, ku, dA, ldab, strideA, dipiv, strideP, dinfo, batch, true)) return r;
+    return run_trf(m, n, kl, ku, Strided<double>{dA, strideA}, ldab, Strided<int>{dipiv, strideP}, dinfo, batch,
+                   (cudaStream_t)stream, variant);
+}
+
+int dgbtrf_strided_batched(int m, int n, int kl, int ku, double *dA, int ldab, int64_t strideA, int *dipiv,
+                           int64_t strideP, int *dinfo, int batch, bandlu_stream_t stream) {
+    return dgbtrf_strided_batched_ex(m, n, kl, ku, dA, ldab, strideA, dipiv, strideP, dinfo, batch, stream,
+                                     BANDLU_AUTO);
+}
+
+int dgbtrf_batched(int m, int n, int kl, int ku, double *const *dA_array, int ldab, int *const *dipiv_array,
+                   int *dinfo, int batch, bandlu_stream_t stream) {
+    if (int r = check_trf(m, n, kl, ku, dA_array, ldab, 0, dipiv_array, 0, dinfo, batch, false)) return r;
+    return run_trf(m, n, kl, ku, PtrArray<double>{dA_array}, ldab, PtrArray<int>{dipiv_array}, dinfo, batch,
+                   (cudaStream_t)stream, BANDLU_AUTO);
+}
+
+int dgbtrs_strided_batched_ex(char trans, int n, int kl, int ku, int nrhs, const double *dA, int ldab,
+                              int64_t strideA, const int *dipiv, int64_t strideP, double *dB, int ldb,
+                              int64_t strideB, int batch, bandlu_stream_t stream, int variant) {
+    if (int r = check_trs(trans, n, kl, ku, nrhs, dA, ldab, strideA, dipiv, strideP, dB, ldb, strideB, batch, true))
+        return r;
+    return run_trs(n, kl, ku, nrhs, Strided<const double>{dA, strideA}, ldab, Strided<const int>{dipiv, strideP},
+                   Strided<double>{dB, strideB}, ldb, nullptr, batch, (cudaStream_t)stream, variant);
+}
+
+int dgbtrs_strided_batched(char trans, int n, int kl, int ku, int nrhs, const double *dA, int ldab,
+                           int64_t strideA, const int *dipiv, int64_t strideP, double *dB, int ldb, int64_t strideB,
+                           int batch, bandlu_stream_t stream) {
+    return dgbtrs_strided_batched_ex(trans, n, kl, ku, nrhs, dA, ldab, strideA, dipiv, strideP, dB, ldb, strideB,
+                                     batch, stream, BANDLU_AUTO);
+}
+
+int dgbtrs_batched(char trans, int n, int kl, int ku, int nrhs, const double *const *dA_array, int ldab,
+                   const int *const *dipiv_array, double *const *dB_array, int ldb, int batch,
+                   bandlu_stream_t stream) {
+    if (int r = check_trs(trans, n, kl, ku, nrhs, dA_array, ldab, 0, dipiv_array, 0, dB_array, ldb, 0, batch, false))
+        return r;
+    return run_trs(n, kl, ku, nrhs, PtrArray<const double>{dA_array}, ldab, PtrArray<const int>{dipiv_array},
+                   PtrArray<double>{dB_array}, ldb, nullptr, batch, (cudaStream_t)stream, BANDLU_AUTO);
+}
+
+int dgbsv_strided_batched(int n, int kl, int ku, int nrhs, double *dA, int ldab, int64_t strideA, int *dipiv,
+                          int64_t strideP, double *dB, int ldb, int64_t strideB, int *dinfo, int batch,
+                          bandlu_stream_t stream) {
+    // (n,kl,ku,nrhs,dA,ldab,strideA,dipiv,strideP,dB,ldb,strideB,dinfo,batch)
+    if (n < 0) return -1;
+    if (kl < 0) return -2;
+    if (ku < 0) return -3;
+    if (nrhs < 0) return -4;
+    if (ldab < 2 * kl + ku + 1) return -6;
+    if (ldb < (n > 1 ? n : 1)) return -11;
+    if (batch < 0) return -14;
+    if (batch > 0) {
+        if (!dA) return -5;
+        if (strideA < (int64_t)ldab * n) return -7;
+        if (!dipiv && n > 0) return -8;
+        if (strideP < n) return -9;
+        if (!dB && n > 0 && nrhs > 0) return -10;
+        if (strideB < (int64_t)ldb * nrhs) return -12;
+        if (!dinfo) return -13;
+    }
+    cudaStream_t st = (cudaStream_t)stream;
+    if (int r = run_trf(n, n, kl, ku, Strided<double>{dA, strideA}, ldab, Strided<int>{dipiv, strideP}, dinfo, batch,
+                        st, BANDLU_AUTO))
+        return r;
+    return run_trs(n, kl, ku, nrhs, Strided<const double>{dA, strideA}, ldab, Strided<const int>{dipiv, strideP},
+                   Strided<double>{dB, strideB}, ldb, dinfo, batch, st, BANDLU_AUTO);
+}
+
+int dgbsv_batched(int n, int kl, int ku, int nrhs, double *const *dA_array, int ldab, int *const *dipiv_array,
+                  double *const *dB_array, int ldb, int *dinfo, int batch, bandlu_stream_t stream) {
+    // (n,kl,ku,nrhs,dA_array,ldab,dipiv_array,dB_array,ldb,dinfo,batch)
+    if (n < 0) return -1;
+    if (kl < 0) return -2;
+    if (ku < 0) return -3;
+    if (nrhs < 0) return -4;
+    if (ldab < 2 * kl + ku + 1) return -6;
+    if (ldb < (n > 1 ? n : 1)) return -9;
+    if (batch < 0) return -11;
+    if (batch > 0) {
+        if (!dA_array) return -5;
+        if (!dipiv_array && n > 0) return -7;
+        if (!dB_array && n > 0 && nrhs > 0) return -8;
+        if (!dinfo) return -10;
+    }
+    cudaStream_t st = (cudaStream_t)stream;
+    if (int r = run_trf(n, n, kl, ku, PtrArray<double>{dA_array}, ldab, PtrArray<int>{dipiv_array}, dinfo, batch, st,
+                        BANDLU_AUTO))
+        return r;
+    return run_trs(n, kl, ku, nrhs, PtrArray<const double>{(const double *const *)dA_array}, ldab,
+                   PtrArray<const int>{(const int *const *)dipiv_array}, PtrArray<double>{dB_array}, ldb, dinfo,
+                   batch, st, BANDLU_AUTO);
+}
+
+}  // extern "C"
+
+// ============================================= host-buffer end-to-end path
+// Pipelined over batch chunks on two internal streams: H2D(A_c, B_c) ->
+// gbtrf -> gbtrs -> D2H(A_c, ipiv_c, B_c, info_c); chunk c+1's copies overlap
+// chunk c's kernels (separate copy engines for each direction).
+extern "C" int dgbsv_strided_batched_host(int n, int kl, int ku, int nrhs, double *hA, int ldab, int64_t strideA,
+                                          int *hipiv, int64_t strideP, double *hB, int ldb, int64_t strideB,
+                                          int *hinfo, int batch, bandlu_stream_t stream) {
+    if (n < 0) return -1;
+    if (kl < 0) return -2;
+    if (ku < 0) return -3;
+    if (nrhs < 0) return -4;
+    if (ldab < 2 * kl + ku + 1) return -6;
+    if (ldb < (n > 1 ? n : 1)) return -11;
+    if (batch < 0) return -14;
+    if (batch == 0) return 0;
+    if (!hA) return -5;
+    if (strideA < (int64_t)ldab * n) return -7;
+    if (!hipiv && n > 0) return -8;
+    if (strideP < n) return -9;
+    if (!hB && n > 0 && nrhs > 0) return -10;
+    if (strideB < (int64_t)ldb * nrhs) return -12;
+    if (!hinfo) return -13;
+
+    cudaStream_t user = (cudaStream_t)stream;
+    const int64_t bytes_per = strideA * 8 + strideB * 8 + strideP * 4 + 4;
+    int64_t ch = (int64_t)((256ll << 20) / (bytes_per > 0 ? bytes_per : 1));  // ~256 MB per chunk
+    ch = ch < 1 ? 1 : ch;
+    if (ch > (batch + 3) / 4) ch = (batch + 3) / 4;  // at least ~4 chunks for overlap
+    if (ch < 1) ch = 1;
+    const int nchunks = (int)((batch + ch - 1) / ch);
+
+    cudaError_t e;
+    cudaStream_t s[2] = {nullptr, nullptr};
+    cudaEvent_t ev0 = nullptr, ev[2] = {nullptr, nullptr};
+    double *dA[2] = {nullptr, nullptr}, *dB[2] = {nullptr, nullptr};
+    int *dP[2] = {nullptr, nullptr}, *dI[2] = {nullptr, nullptr};
+    int ret = 0;
+    auto fail = [&](cudaError_t err) { if (!ret) ret = cuda_ret(err); };
+    for (int i = 0; i < 2; ++i) {
+        if ((e = cudaStreamCreateWithFlags(&s[i], cudaStreamNonBlocking)) != cudaSuccess) fail(e);
+        if ((e = cudaEventCreateWithFlags(&ev[i], cudaEventDisableTiming)) != cudaSuccess) fail(e);
+    }
+    if ((e = cudaEventCreateWithFlags(&ev0, cudaEventDisableTiming)) != cudaSuccess) fail(e);
+    if (!ret) {
+        cudaEventRecord(ev0, user);
+        for (int i = 0; i < 2 && !ret; ++i) {
+            cudaStreamWaitEvent(s[i], ev0, 0);
+            if ((e = cudaMallocAsync((void **)&dA[i], (size_t)(ch * strideA * 8), s[i])) != cudaSuccess) fail(e);
+            if ((e = cudaMallocAsync((void **)&dB[i], (size_t)(ch * strideB * 8 + 8), s[i])) != cudaSuccess) fail(e);
+            if ((e = cudaMallocAsync((void **)&dP[i], (size_t)(ch * strideP * 4 + 4), s[i])) != cudaSuccess) fail(e);
+            if ((e = cudaMallocAsync((void **)&dI[i], (size_t)(ch * 4), s[i])) != cudaSuccess) fail(e);
+        }
+    }
+    for (int c = 0; c < nchunks && !ret; ++c) {
+        const int i = c & 1;
+        const int64_t b0 = (int64_t)c * ch;
+        const int cb = (int)((batch - b0) < ch ? (batch - b0) : ch);
+        const size_t aN = (size_t)((cb - 1) * strideA + (int64_t)ldab * n);
+        const size_t bN = (size_t)((cb - 1) * strideB + (int64_t)ldb * nrhs);
+        const size_t pN = (size_t)((cb - 1) * strideP + n);
+        cudaMemcpyAsync(dA[i], hA + b0 * strideA, aN * 8, cudaMemcpyHostToDevice, s[i]);
+        if (bN) cudaMemcpyAsync(dB[i], hB + b0 * strideB, bN * 8, cudaMemcpyHostToDevice, s[i]);
+        int r = dgbsv_strided_batched(n, kl, ku, nrhs, dA[i], ldab, strideA, dP[i], strideP, dB[i], ldb, strideB,
+                                      dI[i], cb, (bandlu_stream_t)s[i]);
+        if (r) { ret = r; break; }
+        cudaMemcpyAsync(hA + b0 * strideA, dA[i], aN * 8, cudaMemcpyDeviceToHost, s[i]);
+        if (pN && n > 0) cudaMemcpyAsync(hipiv + b0 * strideP, dP[i], pN * 4, cudaMemcpyDeviceToHost, s[i]);
+        if (bN) cudaMemcpyAsync(hB + b0 * strideB, dB[i], bN * 8, cudaMemcpyDeviceToHost, s[i]);
+        cudaMemcpyAsync(hinfo + b0, dI[i], (size_t)cb * 4, cudaMemcpyDeviceToHost, s[i]);
+        if ((e = cudaGetLastError()) != cudaSuccess) fail(e);
+    }
+    for (int i = 0; i < 2; ++i) {
+        if (s[i]) {
+            if (dA[i]) cudaFreeAsync(dA[i], s[i]);
+            if (dB[i]) cudaFreeAsync(dB[i], s[i]);
+            if (dP[i]) cudaFreeAsync(dP[i], s[i]);
+            if (dI[i]) cudaFreeAsync(dI[i], s[i]);
+            cudaEventRecord(ev[i], s[i]);
+            cudaStreamWaitEvent(user, ev[i], 0);
+        }
+    }
+    if ((e = cudaStreamSynchronize(user)) != cudaSuccess) fail(e);
+    for (int i = 0; i < 2; ++i) {
+        if (s[i]) cudaStreamDestroy(s[i]);
+        if (ev[i]) cudaEventDestroy(ev[i]);
+    }
+    if (ev0) cudaEventDestroy(ev0);
+    return ret;
+}

@@ -1,0 +1,125 @@
+"""C-ABI boundary tests that need no GPU: the shared library loads, exports
+every symbol include/bandlu.h declares, and rejects illegal arguments with
+LAPACK-numbered codes before touching the device (no compute calls here)."""
+import ctypes
+import os
+import re
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HDR = os.path.join(ROOT, "include", "bandlu.h")
+
+
+@pytest.fixture(scope="module")
+def lib():
+    from paper_conf_sc_abdelfattahtlad23_b200 import _build, binding
+    _build.build()  # nvcc cross-compiles sm_100a without a GPU
+    return binding.load()
+
+
+def declared_functions():
+    txt = open(HDR).read()
+    txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
+    return sorted(set(re.findall(r"^\s*int\s+(\w+)\s*\(", txt, flags=re.M)))
+
+
+def test_header_declares_the_boundary():
+    names = declared_functions()
+    for n in ("dgbtrf_batched", "dgbtrf_strided_batched", "dgbtrs_batched", "dgbtrs_strided_batched",
+              "dgbsv_batched", "dgbsv_strided_batched", "dgbsv_strided_batched_host"):
+        assert n in names
+
+
+def test_library_exports_every_declared_symbol(lib):
+    from paper_conf_sc_abdelfattahtlad23_b200 import binding
+    for name in declared_functions():
+        assert hasattr(lib, name), name
+    assert set(declared_functions()) <= set(binding.EXPORTS)
+    assert lib.bandlu_version() >= 1
+
+
+NULL = ctypes.c_void_p(0)
+FAKE = ctypes.c_void_p(0x1000)  # never dereferenced: every case below fails argument checking
+
+
+def test_trf_argument_errors(lib):
+    f = lib.dgbtrf_strided_batched
+    # (m, n, kl, ku, dA, ldab, strideA, dipiv, strideP, dinfo, batch, stream)
+    assert f(-1, 4, 1, 1, FAKE, 4, 16, FAKE, 4, FAKE, 1, NULL) == -1
+    assert f(4, -1, 1, 1, FAKE, 4, 16, FAKE, 4, FAKE, 1, NULL) == -2
+    assert f(4, 4, -1, 1, FAKE, 4, 16, FAKE, 4, FAKE, 1, NULL) == -3
+    assert f(4, 4, 1, -1, FAKE, 4, 16, FAKE, 4, FAKE, 1, NULL) == -4
+    assert f(4, 4, 1, 1, FAKE, 3, 16, FAKE, 4, FAKE, 1, NULL) == -6  # ldab < 2kl+ku+1
+    assert f(4, 4, 1, 1, NULL, 4, 16, FAKE, 4, FAKE, 1, NULL) == -5
+    assert f(4, 4, 1, 1, FAKE, 4, 15, FAKE, 4, FAKE, 1, NULL) == -7
+    assert f(4, 4, 1, 1, FAKE, 4, 16, NULL, 4, FAKE, 1, NULL) == -8
+    assert f(4, 4, 1, 1, FAKE, 4, 16, FAKE, 3, FAKE, 1, NULL) == -9
+    assert f(4, 4, 1, 1, FAKE, 4, 16, FAKE, 4, NULL, 1, NULL) == -10
+    assert f(4, 4, 1, 1, FAKE, 4, 16, FAKE, 4, FAKE, -1, NULL) == -11
+    assert f(4, 4, 1, 1, NULL, 4, 16, NULL, 4, NULL, 0, NULL) == 0  # batch 0: quick return, no launch
+    g = lib.dgbtrf_batched  # LAPACK numbering
+    assert g(4, 4, 1, 1, FAKE, 3, FAKE, FAKE, 1, NULL) == -6
+    assert g(4, 4, 1, 1, FAKE, 4, FAKE, NULL, 1, NULL) == -8
+    assert g(4, 4, 1, 1, FAKE, 4, FAKE, FAKE, -2, NULL) == -9
+
+
+def test_trs_argument_errors(lib):
+    f = lib.dgbtrs_strided_batched
+    # (trans, n, kl, ku, nrhs, dA, ldab, strideA, dipiv, strideP, dB, ldb, strideB, batch, stream)
+    ok = dict(n=4, kl=1, ku=1, nrhs=1, ldab=4, sA=16, sP=4, ldb=4, sB=4)
+
+    def call(trans=b"N", **kw):
+        a = dict(ok, **kw)
+        return f(trans, a["n"], a["kl"], a["ku"], a["nrhs"], FAKE, a["ldab"], a["sA"], FAKE, a["sP"], FAKE,
+                 a["ldb"], a["sB"], kw.get("batch", 1), NULL)
+    assert call(trans=b"X") == -1
+    assert call(n=-1) == -2
+    assert call(kl=-1) == -3
+    assert call(ku=-1) == -4
+    assert call(nrhs=-1) == -5
+    assert call(ldab=3) == -7
+    assert call(sA=15) == -8
+    assert call(sP=3) == -10
+    assert call(ldb=3) == -12
+    assert call(sB=3) == -13
+    assert call(batch=-1) == -14
+    assert call(trans=b"T") == 1000  # transposed solve not implemented yet
+    g = lib.dgbtrs_batched  # (trans,n,kl,ku,nrhs,A,ldab,P,B,ldb,batch,stream): LAPACK numbering
+    assert g(b"N", 4, 1, 1, 1, FAKE, 4, FAKE, FAKE, 3, 1, NULL) == -10
+    assert g(b"N", 4, 1, 1, 1, FAKE, 4, NULL, FAKE, 4, 1, NULL) == -8
+
+
+def test_gbsv_argument_errors(lib):
+    g = lib.dgbsv_batched  # (n,kl,ku,nrhs,A,ldab,P,B,ldb,info,batch,stream) -- LAPACK DGBSV numbering
+    assert g(-1, 1, 1, 1, FAKE, 4, FAKE, FAKE, 4, FAKE, 1, NULL) == -1
+    assert g(4, -1, 1, 1, FAKE, 4, FAKE, FAKE, 4, FAKE, 1, NULL) == -2
+    assert g(4, 1, -1, 1, FAKE, 4, FAKE, FAKE, 4, FAKE, 1, NULL) == -3
+    assert g(4, 1, 1, -1, FAKE, 4, FAKE, FAKE, 4, FAKE, 1, NULL) == -4
+    assert g(4, 1, 1, 1, FAKE, 3, FAKE, FAKE, 4, FAKE, 1, NULL) == -6
+    assert g(4, 1, 1, 1, FAKE, 4, FAKE, FAKE, 3, FAKE, 1, NULL) == -9
+    assert g(4, 1, 1, 1, FAKE, 4, FAKE, FAKE, 4, NULL, 1, NULL) == -10
+    s = lib.dgbsv_strided_batched
+    assert s(4, 1, 1, 1, FAKE, 4, 16, FAKE, 4, FAKE, 3, 4, FAKE, 1, NULL) == -11
+    h = lib.dgbsv_strided_batched_host
+    assert h(4, 1, 1, 1, FAKE, 4, 16, FAKE, 4, FAKE, 4, 4, NULL, 1, NULL) == -13
+
+
+def test_variant_heuristic_is_shape_only(lib):
+    from paper_conf_sc_abdelfattahtlad23_b200 import binding as b
+    assert b.trf_variant(512, 512, 10, 10) == b.WINDOW
+    assert b.trf_variant(256, 256, 1, 1) == b.WINDOW
+    assert b.trf_variant(100, 100, 32, 32) == b.GENERIC  # kl+1 > 32 lanes: safeguard kernel
+    assert b.trf_variant(0, 5, 1, 1) == b.GENERIC
+    assert b.trs_variant(1024, 2, 32, 16) == b.WINDOW
+
+
+def test_product_package_does_not_import_oracle():
+    """The product path must not route through the oracle (task ③)."""
+    pkg = os.path.join(ROOT, "paper_conf_sc_abdelfattahtlad23_b200")
+    for dirpath, _, files in os.walk(pkg):
+        for fn in files:
+            if fn.endswith((".py", ".cu", ".cuh", ".h")):
+                txt = open(os.path.join(dirpath, fn)).read()
+                assert "import oracle" not in txt and "from oracle" not in txt, fn
+                assert "bandlu_oracle" not in txt and "liboracle" not in txt, fn

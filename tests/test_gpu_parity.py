@@ -1,0 +1,252 @@
+"""GPU parity: the sm_100a path (through the C ABI) vs the CPU oracle,
+element by element on the same seeded inputs (task ③).
+
+Bar (BASELINE.json north_star): ipiv and info bit-exact; factors within
+1e-12 max relative entrywise error -- and since the kernels execute the
+oracle's exact fp64 operation sequence we assert the stronger `==` equality
+(signed zeros compare equal) plus an identical NaN pattern over
+the WHOLE band array (fill rows, corners and padding rows carry NaN
+sentinels, so any stray read or write shows up); solutions likewise, and the
+scaled backward error <= 10.
+"""
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_sc_abdelfattahtlad23_b200 import inputs as I
+from tests.bandref import backward_error, band_to_dense, same_bits
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import paper_conf_sc_abdelfattahtlad23_b200 as bl  # noqa: E402
+
+WINDOW_BANDS = [(0, 0), (0, 3), (1, 1), (2, 2), (2, 3), (3, 0), (3, 2), (4, 4), (10, 7), (10, 10), (2, 32)]
+
+
+def _gpu_trf(A_np, m, n, kl, ku, variant=bl.AUTO):
+    A = torch.from_numpy(A_np).cuda()
+    batch = A.shape[0]
+    ipiv = torch.zeros((batch, max(min(m, n), 1)), dtype=torch.int32, device="cuda")
+    info = torch.full((batch,), -7, dtype=torch.int32, device="cuda")
+    bl.dgbtrf_strided_batched(m, n, kl, ku, A, ipiv, info, variant=variant)
+    torch.cuda.synchronize()
+    return A.cpu().numpy(), ipiv.cpu().numpy()[:, :min(m, n)], info.cpu().numpy()
+
+
+def _check_trf(m, n, kl, ku, batch, variant, ldab=None, first=0, A_in=None):
+    A0 = I.gen_band(m, n, kl, ku, ldab=ldab, count=batch, first=first) if A_in is None else A_in
+    Ao = A0.copy()
+    ipo, info_o = oracle.dgbtrf(Ao, m, n, kl, ku)
+    Ag, ipg, info_g = _gpu_trf(A0, m, n, kl, ku, variant)
+    assert np.array_equal(info_g, info_o)
+    assert np.array_equal(ipg, ipo)
+    bad = ~same_bits(Ag, Ao)
+    assert not bad.any(), f"{bad.sum()} mismatching band entries, first at {np.argwhere(bad)[0]}"
+    return Ao, ipo, info_o
+
+
+@pytest.mark.parametrize("kl,ku", WINDOW_BANDS)
+@pytest.mark.parametrize("variant", [bl.WINDOW, bl.GENERIC])
+@pytest.mark.parametrize("n", [1, 2, 7, 37, 100])
+def test_trf_parity_small(kl, ku, variant, n):
+    # ragged batch (not a multiple of matrices per warp / block)
+    _check_trf(n, n, kl, ku, batch=37, variant=variant)
+
+
+@pytest.mark.parametrize("kl,ku", WINDOW_BANDS)
+@pytest.mark.parametrize("mn", [(30, 20), (20, 30), (5, 40), (40, 5), (1, 9), (9, 1)])
+def test_trf_parity_rectangular(kl, ku, mn):
+    m, n = mn
+    for variant in (bl.WINDOW, bl.GENERIC):
+        _check_trf(m, n, kl, ku, batch=9, variant=variant)
+
+
+@pytest.mark.parametrize("kl,ku", [(2, 3), (10, 10), (5, 9), (33, 20), (32, 32), (40, 64), (0, 40)])
+def test_trf_parity_generic_any_band(kl, ku):
+    _check_trf(150, 150, kl, ku, batch=11, variant=bl.GENERIC)
+    assert bl.trf_variant(150, 150, kl, ku) in (bl.GENERIC, bl.WINDOW)
+
+
+@pytest.mark.parametrize("kl,ku", [(1, 1), (10, 10), (2, 32)])
+def test_trf_parity_padded_ldab(kl, ku):
+    ldab = 2 * kl + ku + 1 + 3  # extra NaN rows at the bottom stay untouched
+    for variant in (bl.WINDOW, bl.GENERIC):
+        _check_trf(70, 70, kl, ku, batch=5, variant=variant, ldab=ldab)
+
+
+@pytest.mark.parametrize("kl,ku", [(1, 1), (2, 3), (10, 10), (2, 32), (0, 3), (3, 0)])
+def test_trf_parity_planted_zero_pivots(kl, ku):
+    n = 60
+    A = I.gen_band(n, n, kl, ku, count=6)
+    kv = kl + ku
+    for b, z in enumerate([1, 2, 30, 59, 60, 45]):
+        col = A[b, z - 1, kl:kv + kl + 1]
+        A[b, z - 1, kl:kv + kl + 1] = np.where(np.isnan(col), np.nan, 0.0)
+    A[5, 10, kl:kv + kl + 1] = np.where(np.isnan(A[5, 10, kl:kv + kl + 1]), np.nan, 0.0)  # two zeros
+    for variant in (bl.WINDOW, bl.GENERIC):
+        Ao, ipo, info = _check_trf(n, n, kl, ku, 6, variant, A_in=A.copy())
+        assert list(info) == [1, 2, 30, 59, 60, 11]
+
+
+@pytest.mark.parametrize("kl,ku", [(1, 1), (2, 2), (10, 10), (2, 32)])
+def test_trf_parity_exact_ties(kl, ku):
+    """Integer-valued bands with many exact |pivot| ties: both sides take the
+    same decision (first index, Q2) in the same precision."""
+    n = 64
+    A = I.gen_band(n, n, kl, ku, count=16)
+    A = np.where(np.isnan(A), np.nan, np.sign(A) * np.ceil(np.abs(A) * 2.0))  # values in {+-1, +-2}
+    for variant in (bl.WINDOW, bl.GENERIC):
+        _check_trf(n, n, kl, ku, 16, variant, A_in=A.copy())
+
+
+def _gpu_trs(Af, ipiv, B_np, n, kl, ku, variant=bl.AUTO):
+    A = torch.from_numpy(Af).cuda()
+    P = torch.from_numpy(np.ascontiguousarray(ipiv.astype(np.int32))).cuda()
+    B = torch.from_numpy(B_np).cuda()
+    bl.dgbtrs_strided_batched("N", n, kl, ku, A, P, B, variant=variant)
+    torch.cuda.synchronize()
+    return B.cpu().numpy()
+
+
+@pytest.mark.parametrize("kl,ku", WINDOW_BANDS)
+@pytest.mark.parametrize("nrhs", [1, 2, 3, 16, 33])
+@pytest.mark.parametrize("variant", [bl.WINDOW, bl.GENERIC])
+def test_trs_parity(kl, ku, nrhs, variant):
+    n, batch = 45, 13
+    A = I.gen_band(n, n, kl, ku, count=batch)
+    ipiv, info = oracle.dgbtrf(A, n, n, kl, ku)
+    assert np.all(info == 0)
+    B = I.gen_rhs(n, nrhs, ldb=n + 2, count=batch)
+    Bo = B.copy()
+    oracle.dgbtrs(A, ipiv, Bo, n, kl, ku)
+    Bg = _gpu_trs(A, ipiv, B, n, kl, ku, variant)
+    assert np.all(same_bits(Bg, Bo))
+
+
+@pytest.mark.parametrize("n", [1, 2, 3, 8, 9, 130])
+@pytest.mark.parametrize("kl,ku", [(1, 1), (10, 10), (2, 32), (0, 0)])
+def test_trs_parity_sizes(n, kl, ku):
+    A = I.gen_band(n, n, kl, ku, count=7)
+    ipiv, info = oracle.dgbtrf(A, n, n, kl, ku)
+    B = I.gen_rhs(n, 2, count=7)
+    Bo = B.copy()
+    oracle.dgbtrs(A, ipiv, Bo, n, kl, ku)
+    for variant in (bl.WINDOW, bl.GENERIC):
+        assert np.all(same_bits(_gpu_trs(A, ipiv, B.copy(), n, kl, ku, variant), Bo))
+
+
+@pytest.mark.parametrize("kl,ku,nrhs", [(2, 2, 1), (10, 10, 1), (2, 32, 16), (5, 6, 3)])
+def test_gbsv_parity_with_singular(kl, ku, nrhs):
+    n, batch = 80, 10
+    A = I.gen_band(n, n, kl, ku, count=batch)
+    kv = kl + ku
+    A[3, 17, kl:kv + kl + 1] = np.where(np.isnan(A[3, 17, kl:kv + kl + 1]), np.nan, 0.0)
+    B = I.gen_rhs(n, nrhs, count=batch)
+    Ao, Bo = A.copy(), B.copy()
+    ipo, info_o = oracle.dgbsv(Ao, Bo, n, kl, ku)
+    Ag = torch.from_numpy(A).cuda(); Bg = torch.from_numpy(B).cuda()
+    P = torch.zeros((batch, n), dtype=torch.int32, device="cuda")
+    inf = torch.zeros(batch, dtype=torch.int32, device="cuda")
+    bl.dgbsv_strided_batched(n, kl, ku, Ag, P, Bg, inf)
+    torch.cuda.synchronize()
+    assert np.array_equal(inf.cpu().numpy(), info_o) and info_o[3] == 18
+    assert np.array_equal(P.cpu().numpy(), ipo)
+    assert np.all(same_bits(Ag.cpu().numpy(), Ao))
+    Bgn = Bg.cpu().numpy()
+    assert np.all(same_bits(Bgn, Bo))
+    assert np.array_equal(Bgn[3], B[3])  # untouched where info > 0
+
+
+def test_pointer_array_variants_match_strided():
+    n, kl, ku, nrhs, batch = 50, 10, 10, 2, 9
+    A = I.gen_band(n, n, kl, ku, count=batch)
+    B = I.gen_rhs(n, nrhs, count=batch)
+    Ao, Bo = A.copy(), B.copy()
+    ipo, info_o = oracle.dgbsv(Ao, Bo, n, kl, ku)
+    As = [torch.from_numpy(A[i].copy()).cuda() for i in range(batch)]
+    Bs = [torch.from_numpy(B[i].copy()).cuda() for i in range(batch)]
+    Ps = [torch.zeros(n, dtype=torch.int32, device="cuda") for _ in range(batch)]
+    info = torch.zeros(batch, dtype=torch.int32, device="cuda")
+    ldab = 2 * kl + ku + 1
+    bl.dgbtrf_batched(n, n, kl, ku, bl.ptr_array(As), ldab, bl.ptr_array(Ps), info, batch)
+    bl.dgbtrs_batched("N", n, kl, ku, nrhs, bl.ptr_array(As), ldab, bl.ptr_array(Ps), bl.ptr_array(Bs), n, batch)
+    torch.cuda.synchronize()
+    for i in range(batch):
+        assert np.all(same_bits(As[i].cpu().numpy(), Ao[i]))
+        assert np.array_equal(Ps[i].cpu().numpy(), ipo[i])
+        assert np.all(same_bits(Bs[i].cpu().numpy(), Bo[i]))
+    # and dgbsv_batched
+    As2 = [torch.from_numpy(A[i].copy()).cuda() for i in range(batch)]
+    Bs2 = [torch.from_numpy(B[i].copy()).cuda() for i in range(batch)]
+    bl.dgbsv_batched(n, kl, ku, nrhs, bl.ptr_array(As2), ldab, bl.ptr_array(Ps), bl.ptr_array(Bs2), n, info, batch)
+    torch.cuda.synchronize()
+    for i in range(batch):
+        assert np.all(same_bits(Bs2[i].cpu().numpy(), Bo[i]))
+
+
+def test_host_buffer_gbsv_matches_oracle():
+    n, kl, ku, nrhs, batch = 64, 2, 2, 1, 100  # BASELINE configs[0]
+    A = I.gen_band(n, n, kl, ku, count=batch)
+    B = I.gen_rhs(n, nrhs, count=batch)
+    Ao, Bo = A.copy(), B.copy()
+    ipo, info_o = oracle.dgbsv(Ao, Bo, n, kl, ku)
+    At = torch.from_numpy(A.copy()).pin_memory(); Bt = torch.from_numpy(B.copy()).pin_memory()
+    P = torch.zeros((batch, n), dtype=torch.int32).pin_memory()
+    inf = torch.zeros(batch, dtype=torch.int32).pin_memory()
+    bl.dgbsv_strided_batched_host(n, kl, ku, At, P, Bt, inf)
+    assert np.all(same_bits(At.numpy(), Ao)) and np.all(same_bits(Bt.numpy(), Bo))
+    assert np.array_equal(P.numpy(), ipo) and np.array_equal(inf.numpy(), info_o)
+
+
+def test_quick_returns_write_info():
+    A = torch.zeros((5, 3, 4), dtype=torch.float64, device="cuda")
+    ipiv = torch.zeros((5, 1), dtype=torch.int32, device="cuda")
+    info = torch.full((5,), 9, dtype=torch.int32, device="cuda")
+    bl.dgbtrf_strided_batched(0, 3, 1, 1, A, ipiv, info)
+    torch.cuda.synchronize()
+    assert torch.all(info == 0)
+    assert torch.all(A == 0)
+
+
+# ---------------------------------------------- full-size sampled parity
+# BASELINE.json configs at full batch size, launched exactly as bench.py does
+# (AUTO variant, strided, one trf + one trs launch); the oracle recomputes a
+# sample of matrices one by one from the same seeded generator.
+FULL = [  # (batch, n, kl, ku, nrhs)
+    (100, 64, 2, 2, 1),
+    (10000, 256, 1, 1, 1),
+    (10000, 512, 10, 10, 1),
+    (5000, 1024, 2, 32, 16),
+]
+
+
+@pytest.mark.parametrize("batch,n,kl,ku,nrhs", FULL)
+def test_full_size_sampled_parity(batch, n, kl, ku, nrhs):
+    A = torch.from_numpy(I.gen_band(n, n, kl, ku, count=batch)).cuda()
+    B = torch.from_numpy(I.gen_rhs(n, nrhs, count=batch)).cuda()
+    P = torch.zeros((batch, n), dtype=torch.int32, device="cuda")
+    info = torch.zeros(batch, dtype=torch.int32, device="cuda")
+    bl.dgbtrf_strided_batched(n, n, kl, ku, A, P, info)
+    bl.dgbtrs_strided_batched("N", n, kl, ku, A, P, B)
+    torch.cuda.synchronize()
+    rng = np.random.default_rng(1)
+    sample = np.unique(np.concatenate([[0, batch - 1], rng.integers(0, batch, 40)]))
+    for i in sample:
+        Ao = I.gen_band(n, n, kl, ku, count=1, first=int(i))
+        Bo = I.gen_rhs(n, nrhs, count=1, first=int(i))
+        A0, B0 = Ao.copy(), Bo.copy()
+        ipo, info_o = oracle.dgbtrf(Ao, n, n, kl, ku)
+        oracle.dgbtrs(Ao, ipo, Bo, n, kl, ku)
+        assert info[i].item() == info_o[0]
+        assert np.array_equal(P[i].cpu().numpy(), ipo[0])
+        assert np.all(same_bits(A[i].cpu().numpy(), Ao[0]))
+        Bi = B[i].cpu().numpy()
+        assert np.all(same_bits(Bi, Bo[0]))
+        if i == sample[0]:
+            D = band_to_dense(A0[0], n, n, kl, ku)
+            assert backward_error(D, Bi[:, :n].T, B0[0][:, :n].T) <= 10.0
+    # properties over the whole batch: pivot range, info
+    j = torch.arange(n, device="cuda", dtype=torch.int32)
+    assert bool(torch.all(P >= j + 1)) and bool(torch.all(P <= torch.clamp(j + 1 + kl, max=n)))
+    assert int(info.abs().sum()) == 0
