@@ -19,6 +19,9 @@ struct PtrArray {
     __device__ __forceinline__ T *get(int64_t i) const { return ptrs[i]; }
 };
 
+// valid global address for zero-filling cp.async (src-size 0 reads nothing)
+__device__ double g_dummy[2];
+
 __device__ __forceinline__ unsigned lane_id() { return threadIdx.x & 31u; }
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
@@ -38,6 +41,63 @@ __device__ __forceinline__ void cp_async4(uint32_t dst, const void *src, uint32_
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory"); }
+
+// Predicated shared-memory moves (no branch / reconvergence; a predicated-off
+// load leaves its destination register unchanged).
+__device__ __forceinline__ void st_shared_f64_if(bool p, uint32_t addr, double v) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %0, 0;\n\t@q st.shared.f64 [%1], %2;\n\t}\n" ::"r"((int)p),
+                 "r"(addr), "d"(v)
+                 : "memory");
+}
+__device__ __forceinline__ void st_shared_s32_if(bool p, uint32_t addr, int v) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %0, 0;\n\t@q st.shared.s32 [%1], %2;\n\t}\n" ::"r"((int)p),
+                 "r"(addr), "r"(v)
+                 : "memory");
+}
+__device__ __forceinline__ void ld_shared_f64_if(bool p, uint32_t addr, double &v) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %1, 0;\n\t@q ld.shared.f64 %0, [%2];\n\t}\n"
+                 : "+d"(v)
+                 : "r"((int)p), "r"(addr)
+                 : "memory");
+}
+
+// Four predicated 8-byte shared loads / stores under ONE predicate (one asm
+// block so ptxas keeps them predicated instead of branching around each).
+__device__ __forceinline__ void ld4_shared_if(bool p, uint32_t a, double &x0, double &x1, double &x2, double &x3) {
+    asm volatile(
+        "{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %4, 0;\n\t"
+        "@q ld.shared.f64 %0, [%5+%6];\n\t@q ld.shared.f64 %1, [%5+%7];\n\t"
+        "@q ld.shared.f64 %2, [%5+%8];\n\t@q ld.shared.f64 %3, [%5+%9];\n\t}\n"
+        : "+d"(x0), "+d"(x1), "+d"(x2), "+d"(x3)
+        : "r"((int)p), "r"(a), "n"(0), "n"(8), "n"(16), "n"(24)
+        : "memory");
+}
+__device__ __forceinline__ void st4_shared_if(bool p, uint32_t a, double x0, double x1, double x2, double x3) {
+    asm volatile(
+        "{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %0, 0;\n\t"
+        "@q st.shared.f64 [%1+%6], %2;\n\t@q st.shared.f64 [%1+%7], %3;\n\t"
+        "@q st.shared.f64 [%1+%8], %4;\n\t@q st.shared.f64 [%1+%9], %5;\n\t}\n" ::"r"((int)p),
+        "r"(a), "d"(x0), "d"(x1), "d"(x2), "d"(x3), "n"(0), "n"(8), "n"(16), "n"(24)
+        : "memory");
+}
+
+__device__ __forceinline__ void st_shared_v2_if(bool p, uint32_t a, double2 v) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %0, 0;\n\t@q st.shared.v2.f64 [%1], {%2, %3};\n\t}\n" ::"r"(
+                     (int)p),
+                 "r"(a), "d"(v.x), "d"(v.y)
+                 : "memory");
+}
+__device__ __forceinline__ void ld_shared_v2_if(bool p, uint32_t a, double2 &v) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %2, 0;\n\t@q ld.shared.v2.f64 {%0, %1}, [%3];\n\t}\n"
+                 : "+d"(v.x), "+d"(v.y)
+                 : "r"((int)p), "r"(a)
+                 : "memory");
+}
+__device__ __forceinline__ double ld_shared_f64(uint32_t a) {
+    double v;
+    asm volatile("ld.shared.f64 %0, [%1];\n" : "=d"(v) : "r"(a) : "memory");
+    return v;
+}
 
 // |x| as an ordered integer key: for non-negative doubles the IEEE bit
 // pattern orders like the value (used for the exact pivot search).

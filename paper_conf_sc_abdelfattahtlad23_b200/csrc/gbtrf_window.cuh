@@ -13,23 +13,28 @@
 //  * A group of G = pow2 >= KL+1 lanes owns one matrix; 32/G matrices share a
 //    warp (per-warp instruction cost is shared by all of them).
 //  * Row-owner mapping: each of the KL+1 active lanes holds ONE row of the
-//    active window -- the KV+1 = KL+KU+1 values at columns j..j+KV -- in
-//    registers.  Columns map to register slots (col mod W) and the step loop
-//    is unrolled W times, so no register ever moves when the window slides.
+//    active window -- the W = KL+KU+1 values at columns j..j+KV -- in
+//    registers, column c in slot c mod W, slots paired into double2 so rows
+//    move to/from shared memory with 128-bit accesses.  The column loop is
+//    unrolled W times: sliding the window never moves a register.
 //  * Row interchanges are relabelings: a lane carries the logical position of
 //    its row.  LAPACK swaps only columns j..ju; beyond ju both rows hold
 //    structural zeros, so swapping whole rows is identical.
-//  * IAMAX: exact first-max via three redux.sync over the 64-bit |x| key and
-//    the logical position (ties -> smallest position, Q2).
-//  * The pivot row (U row j) goes through a 16-byte-aligned smem record that
-//    is the broadcast source for the rank-1 update (FP64 FMA in registers)
-//    and the source of the U-row store to HBM.  Multipliers are stored by
-//    their owning lanes.  Each step thus needs one __syncwarp.
-//  * Input rows are gathered by cp.async (LDGSTS, L1-allocating, zero-fill
-//    outside the matrix) into a 2-batch row ring in smem, NR rows ahead of
-//    use; the lane freed by the pivot row reloads its registers from it.
-//  * Every input element is read from HBM once and every output element is
-//    written once; the fill rows (input) are never read.
+//  * IAMAX: butterfly max of the high word of the |x| bit pattern + ballot;
+//    exact slow path (low word, then smallest logical row) only when the
+//    high words tie (zero pivots, exact ties) -- first-max semantics (Q2).
+//  * The pivot row is broadcast to its group with width-G shuffles (the
+//    shuffle path runs beside the shared-memory pipe, which the row staging
+//    and the U store use); every lane then applies the rank-1 update with
+//    FP64 FMAs in registers.  The pivot lane also drops its row (= U row j)
+//    into a double-buffered smem record that the group stores to HBM one
+//    step later.  Multipliers are stored by their owning lanes.
+//  * Input rows are gathered one row per step by cp.async (LDGSTS,
+//    L1-allocating, zero-fill outside the matrix) into a 16-row smem ring in
+//    slot order, D = 8 rows ahead; the lane freed by the pivot row reloads
+//    its registers from it with 128-bit loads.  Fill rows (input) are never
+//    read; every input element is read from HBM once, every output element
+//    written once.
 #pragma once
 #include "common.cuh"
 
@@ -38,152 +43,198 @@ namespace bandlu {
 template <int KL_, int KU_>
 struct TrfWin {
     static constexpr int KL = KL_, KU = KU_, KV = KL + KU, W = KV + 1;
+    static constexpr int U = 4;                  // columns per unrolled block (window shift granularity)
+    static constexpr int WS = W + U;             // register slots: column j0 + r in slot r during a block
+    static constexpr int H = (WS + 1) / 2;       // double2 slot pairs
+    static constexpr int WP = 2 * H + 2;         // record / ring-row pitch in doubles (16 B rows, +1 free slot)
     static constexpr int G = pow2_ceil(KL + 1);  // lanes per matrix
     static constexpr int GPW = 32 / G;           // matrices per warp
-    static constexpr int WP = (W + 1) & ~1;      // even row pitch (doubles) -> 16 B aligned rows
-    static constexpr int NR = W <= 24 ? 8 : 4;   // rows per staging batch (power of 2)
-    static constexpr int RR = 2 * NR;            // ring rows (2 batches)
-    static constexpr int GROUP_DBL = (RR + 2) * WP;  // ring + 2 pivot-row records
-    static constexpr int STAGE_IT = (NR * W + G - 1) / G;
+    static constexpr int D = 8;                  // staging lead (rows)
+    static constexpr int RR = 16;                // ring rows (power of 2, > D, multiple of U)
+    static constexpr int GROUP_DBL = (RR + 2) * WP;  // ring + 2 pivot-row records (double buffered)
+    static constexpr int SIT = (W + G - 1) / G;      // staged elements per lane per row
     static constexpr int WARPS = 4;
+    // register budget: >= 4 CTAs (16 warps) per SM while the window fits
+    static constexpr int MINB = W <= 24 ? 4 : 2;
     static constexpr size_t smem_bytes() { return (size_t)WARPS * GPW * GROUP_DBL * sizeof(double); }
 };
 
 template <int KL, int KU, class AP, class PP>
-__global__ void __launch_bounds__(TrfWin<KL, KU>::WARPS * 32)
+__global__ void __launch_bounds__(TrfWin<KL, KU>::WARPS * 32, TrfWin<KL, KU>::MINB)
     gbtrf_window_kernel(int m, int n, AP A, int ldab, PP P, int *__restrict__ info, int batch) {
     using C = TrfWin<KL, KU>;
-    constexpr int KV = C::KV, W = C::W, G = C::G, WP = C::WP, NR = C::NR, RR = C::RR;
+    constexpr int KV = C::KV, W = C::W, U = C::U, WS = C::WS, H = C::H, G = C::G, WP = C::WP, D = C::D,
+                  RR = C::RR, SIT = C::SIT;
+    static_assert(U % 2 == 0 && RR % U == 0, "block geometry");
     extern __shared__ __align__(16) double smem[];
 
     const int lane = (int)lane_id(), wib = (int)(threadIdx.x >> 5);
     const int g = lane / G, t = lane % G;
     const int64_t mat = ((int64_t)blockIdx.x * C::WARPS + wib) * C::GPW + g;
     const bool live = mat < batch;
-    const unsigned wmask = __ballot_sync(0xffffffffu, live);
-    if (!live) return;
-    const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << (g * G));
+    if (__ballot_sync(0xffffffffu, live) == 0u) return;
+    // Dead groups (batch tail) stay in the warp for the warp-wide shuffles;
+    // they have no candidates, never pivot and never touch global memory.
 
-    double *__restrict__ ab = A.get(mat);
-    int *__restrict__ ipiv = P.get(mat);
+    double *__restrict__ ab = live ? A.get(mat) : nullptr;
+    int *__restrict__ ipiv = live ? P.get(mat) : nullptr;
     if (m <= 0 || n <= 0) {
-        if (t == 0) info[mat] = 0;
+        if (live && t == 0) info[mat] = 0;
         return;
     }
+    const int mloc = live ? m : 0;
     double *ring = smem + (size_t)(wib * C::GPW + g) * C::GROUP_DBL;
-    double *rec = ring + RR * WP;
+    const uint32_t ring_s = smem_u32(ring);
+    const uint32_t rec_s = ring_s + RR * WP * 8;
+    const double *safe = live ? ab : g_dummy;  // zero-fill copies never read it
 
-    // Stage input rows [qb, qb+NR) (row layout: ring[a][c] = A(q, q-KL+c)).
-    auto stage = [&](int b) {
-        const int qb = KL + 1 + b * NR;
-        double *half = ring + (b & 1) * NR * WP;
+    // Ring row of input row q (loaded at step j = q-KL-1, block offset o = j % U)
+    // holds A(q, q-KL+c) at position o+1+c, zeros elsewhere, so one 128-bit
+    // load per slot pair drops it into the window registers.  o is fixed per
+    // ring row (RR % U == 0), so the zero positions are zeroed once here.
+    for (int i = t; i < RR * WP; i += G) ring[i] = 0.0;
+    __syncwarp();
+
+    // ---- staging: lane t copies c = t + k*G (element at AB(KV+KL-c, q-KL+c))
+    int soff[SIT];
 #pragma unroll
-        for (int k = 0; k < C::STAGE_IT; ++k) {
-            const int e = t + k * G;
-            if (e < NR * W) {
-                const int a = e / W, c = e - a * W;
-                const int q = qb + a, col = q - KL + c;
-                const bool ok = (q < m) && (col < n);
-                const double *src = ok ? ab + (int64_t)col * ldab + (KV + KL - c) : ab;
-                cp_async8(smem_u32(half + a * WP + c), src, ok ? 8u : 0u);
+    for (int k = 0; k < SIT; ++k) soff[k] = (t + k * G) * (ldab - 1) + (KV + KL);
+    auto stage_row = [&](int q, const double *rowp) {
+        const uint32_t dst = ring_s + (uint32_t)(((q & (RR - 1)) * WP + 1 + ((q - KL - 1) & (U - 1))) * 8);
+#pragma unroll
+        for (int k = 0; k < SIT; ++k) {
+            const int c = t + k * G;
+            if (c < W) {
+                const bool ok = (q < mloc) && (q - KL + c < n);
+                cp_async8(dst + c * 8, ok ? rowp + soff[k] : safe, ok ? 8u : 0u);
             }
         }
         cp_async_commit();
     };
+#pragma unroll 1
+    for (int d = 0; d < D; ++d) stage_row(KL + 1 + d, live ? ab + (int64_t)(1 + d) * ldab : g_dummy);
+    const double *srow = live ? ab + (int64_t)(1 + D) * ldab : g_dummy;  // &A(q-KL, .) of the row staged next
 
-    // Window registers: v[c % W] = row value at column c, rows 0..KL first.
-    double v[W];
-    int pos = (t <= KL) ? t : 0x7fffffff;
+    // ---- window registers (slot pairs): slot r = column j0 + r; rows 0..KL first
+    double2 v2[H];
+#define VS(k) (((k) & 1) ? v2[(k) >> 1].y : v2[(k) >> 1].x)
 #pragma unroll
-    for (int c = 0; c < W; ++c) {
-        const bool ok = (t <= KL) && (t < m) && (c < n) && (c <= t + KU);
-        v[c] = ok ? ab[(int64_t)c * ldab + (KV + t - c)] : 0.0;
+    for (int h = 0; h < H; ++h) {
+        const int c0 = 2 * h, c1 = 2 * h + 1;
+        const bool ok0 = live && (t <= KL) && (t < m) && (c0 < n) && (c0 <= t + KU);
+        const bool ok1 = live && (t <= KL) && (t < m) && (c1 < n) && (c1 <= t + KU);
+        v2[h].x = ok0 ? ab[(int64_t)c0 * ldab + (KV + t - c0)] : 0.0;
+        v2[h].y = ok1 ? ab[(int64_t)c1 * ldab + (KV + t - c1)] : 0.0;
     }
-    stage(0);
+    int pos = (live && t <= KL) ? t : 0x7fffffff;  // logical row held by this lane
 
     int linfo = 0;
     const int mn = min(m, n);
-    for (int j0 = 0; j0 < mn; j0 += W) {
+    double *colj = live ? ab + KV : nullptr;  // &AB(KV, j)
+    const unsigned gbits = (G == 32) ? 0xffffffffu : ((1u << G) - 1u);
+    const unsigned gbase = (unsigned)(g * G);
+    int rb = 0;  // pivot-row record buffer of step j (double buffered)
+#pragma unroll 1
+    for (int j0 = 0; j0 < mn; j0 += U) {
 #pragma unroll
-        for (int s = 0; s < W; ++s) {
+        for (int s = 0; s < U; ++s) {  // column j = j0 + s sits in slot s
             const int j = j0 + s;
             if (j >= mn) break;
-            const bool batch_start = (j & (NR - 1)) == 0;
-            if (batch_start) cp_async_wait<0>();
+            cp_async_wait<D - 1>();  // row j+KL+1 landed (this lane's part)
 
             // ---- IAMAX over the candidates (logical rows j..min(j+KL, m-1))
-            const double x = v[s];
-            const bool cand = (t <= KL) && (pos < m);
+            const double x = VS(s);
+            const bool cand = (t <= KL) && (pos < mloc);
             const uint64_t key = cand ? abs_key(x) : 0ull;
-            const unsigned hi = (unsigned)(key >> 32), lo = (unsigned)key;
-            const unsigned mhi = __reduce_max_sync(gmask, hi);
-            const unsigned mlo = __reduce_max_sync(gmask, hi == mhi ? lo : 0u);
-            const bool win = (hi == mhi) && (lo == mlo);
-            const unsigned ppos = __reduce_min_sync(gmask, win ? (unsigned)pos : 0xffffffffu);
-            const bool is_piv = ((unsigned)pos == ppos);
-            const bool zp = (mhi | mlo) == 0u;  // exact zero pivot (all candidates are +-0)
-
-            // ---- pivot row -> smem record (U row j: columns j..j+KV)
-            double *rc = rec + (j & 1) * WP;
-            if (is_piv) {
+            const unsigned hi = (unsigned)(key >> 32);
+            unsigned mhi;
+            if constexpr (C::GPW == 2) {  // two full-warp reductions beat a 4-round butterfly
+                const unsigned m0 = __reduce_max_sync(0xffffffffu, g == 0 ? hi : 0u);
+                const unsigned m1 = __reduce_max_sync(0xffffffffu, g == 1 ? hi : 0u);
+                mhi = g == 0 ? m0 : m1;
+            } else if constexpr (C::GPW == 1) {
+                mhi = __reduce_max_sync(0xffffffffu, hi);
+            } else {
+                mhi = hi;
 #pragma unroll
-                for (int c = 0; c < W; c += 2) {
-                    double2 d;
-                    d.x = v[(s + c) % W];
-                    d.y = (c + 1 < W) ? v[(s + c + 1) % W] : 0.0;
-                    *reinterpret_cast<double2 *>(rc + c) = d;
-                }
-                ipiv[j] = (int)ppos + 1;
+                for (int off = 1; off < G; off <<= 1) mhi = max(mhi, __shfl_xor_sync(0xffffffffu, mhi, off));
             }
-            __syncwarp(wmask);
-            if (batch_start) stage(j / NR + 1);
+            unsigned gb = (__ballot_sync(0xffffffffu, cand && hi == mhi) >> gbase) & gbits;
+            if (__any_sync(0xffffffffu, live && __popc(gb) != 1)) {
+                // exact tie-break: low word, then smallest logical row (first index)
+                const unsigned lo = (unsigned)key;
+                unsigned mlo = (cand && hi == mhi) ? lo : 0u;
+#pragma unroll
+                for (int off = 1; off < G; off <<= 1) mlo = max(mlo, __shfl_xor_sync(0xffffffffu, mlo, off));
+                unsigned pp = (cand && hi == mhi && lo == mlo) ? (unsigned)pos : 0xffffffffu;
+#pragma unroll
+                for (int off = 1; off < G; off <<= 1) pp = min(pp, __shfl_xor_sync(0xffffffffu, pp, off));
+                gb = (__ballot_sync(0xffffffffu, cand && (unsigned)pos == pp) >> gbase) & gbits;
+            }
+            const bool is_piv = (t == __ffs(gb) - 1);  // dead groups: gb = 0, nobody
 
-            if (zp && linfo == 0) linfo = j + 1;
-            // interchange = relabel: the old row j takes the pivot row's place
-            if (pos == j && !is_piv) pos = (int)ppos;
+            // ---- pivot row (U row j: slots s..s+KV) + its logical row -> smem record, 128-bit
+            const uint32_t rcs = rec_s + (uint32_t)(rb * WP * 8);
+            const double *rc = ring + RR * WP + rb * WP;
+#pragma unroll
+            for (int h = s / 2; h <= (s + KV) / 2; ++h) st_shared_v2_if(is_piv, rcs + h * 16, v2[h]);
+            st_shared_s32_if(is_piv, rcs + (WP - 1) * 8, pos);  // pitch WP >= WS+1: last double is free
+            __syncwarp();
+
+            // ---- broadcast read: pivot value and pivot row (128-bit loads), its logical row
+            double2 uu[KV / 2 + 2];
+#pragma unroll
+            for (int h = s / 2; h <= (s + KV) / 2; ++h) uu[h - s / 2] = *reinterpret_cast<const double2 *>(rc + 2 * h);
+#define US(k) ((((k) & 1) ? uu[((k) >> 1) - s / 2].y : uu[((k) >> 1) - s / 2].x))
+            const int ppos = *reinterpret_cast<const int *>(rc + WP - 1);
+            const double p = US(s);
+            const bool zp = (p == 0.0);  // exact zero pivot: all candidates are +-0
+            if (is_piv) ipiv[j] = ppos + 1;
+            if (live && zp && linfo == 0) linfo = j + 1;
+            if (live && pos == j && !is_piv) pos = ppos;  // interchange = relabel
 
             // ---- SCAL: multiplier = x * RN(1/p) (DSCAL(ONE/pivot), Q7)
-            double l = x;
-            if (!zp) {
-                const double r = __drcp_rn(rc[0]);
-                l = __dmul_rn(x, r);
-            }
-            if (cand && !is_piv) ab[(int64_t)j * ldab + (KV + pos - j)] = l;
+            const double r = __drcp_rn(p);
+            const double l = zp ? x : __dmul_rn(x, r);
+            const double lu = zp ? 0.0 : l;  // zero pivot: no update
+            if (cand && !is_piv) colj[pos - j] = l;
 
-            // ---- RANK-1 update of the window (DGER, alpha = -1, FMA)
-            if (!zp) {
+            // ---- RANK-1 update of the window columns j+1..j+KV (DGER, alpha = -1, FMA)
 #pragma unroll
-                for (int c = 0; c < W; c += 2) {  // record padded to WP (even): rc[c+1] exists
-                    const double2 u = *reinterpret_cast<const double2 *>(rc + c);
-                    if (c >= 1) v[(s + c) % W] = __fma_rn(l, -u.x, v[(s + c) % W]);
-                    if (c + 1 < W) v[(s + c + 1) % W] = __fma_rn(l, -u.y, v[(s + c + 1) % W]);
-                }
-            }
+            for (int k = s + 1; k <= s + KV; ++k) VS(k) = __fma_rn(lu, -US(k), VS(k));
+#undef US
 
-            // ---- U row j -> HBM: U(j, j+c) at AB(KV-c, j+c)
+            // ---- U row j -> HBM: U(j, j+c) = record[s + c] at AB(KV-c, j+c)
 #pragma unroll
-            for (int c0 = 0; c0 < W; c0 += G) {
-                const int c = c0 + t;
-                if (c < W && j + c < n) ab[(int64_t)(j + c) * ldab + (KV - c)] = rc[c];
+            for (int k = 0; k < SIT; ++k) {
+                const int c = t + k * G;
+                if (live && c < W && j + c < n) colj[(int64_t)c * (ldab - 1)] = rc[s + c];
             }
+            stage_row(j + KL + 1 + D, srow);
 
-            // ---- slide: the pivot lane takes row j+KL+1; column j leaves all rows
-            if (is_piv) {
-                const int q = j + KL + 1;
-                pos = q;
-                const double *rr = ring + ((q - KL - 1) & (RR - 1)) * WP;
+            // ---- slide: the pivot lane takes row j+KL+1 (ring row pre-positioned at slots s+1..s+W)
+            if (is_piv) pos = j + KL + 1;
+            const uint32_t rr = ring_s + (uint32_t)(((j + KL + 1) & (RR - 1)) * WP * 8);
 #pragma unroll
-                for (int c = 0; c < W; c += 2) {
-                    const double2 d = *reinterpret_cast<const double2 *>(rr + c);
-                    v[(s + 1 + c) % W] = d.x;
-                    if (c + 1 < W) v[(s + 2 + c) % W] = d.y;
-                }
+            for (int h = s / 2; h < H; ++h) ld_shared_v2_if(is_piv, rr + h * 16, v2[h]);
+            colj += ldab;
+            srow += ldab;
+            rb ^= 1;
+        }
+        // shift the window by U columns: slot r <- slot r+U (U even: whole pairs move)
+#pragma unroll
+        for (int h = 0; h < H; ++h) {
+            if (h + U / 2 < H) {
+                v2[h] = v2[h + U / 2];
             } else {
-                v[s] = 0.0;
+                v2[h].x = 0.0;
+                v2[h].y = 0.0;
             }
         }
     }
     cp_async_wait<0>();
+#undef VS
+    if (!live) return;
 
     // LAPACK's SET_FILLIN also zeroes fill-row positions whose matrix row is
     // >= m when m < n (those rows are never pivot rows here).

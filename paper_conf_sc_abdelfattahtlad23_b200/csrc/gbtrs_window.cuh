@@ -28,9 +28,6 @@
 
 namespace bandlu {
 
-// valid global address for zero-filling cp.async (src-size 0 reads nothing)
-__device__ double g_dummy[2];
-
 template <int KL_, int KU_>
 struct TrsWin {
     static constexpr int KL = KL_, KU = KU_, KV = KL + KU;

@@ -1,0 +1,30 @@
+"""One hot-path step (dgbtrf + dgbtrs) at a BASELINE config, for ncu captures.
+
+  python tools/prof_step.py C3 [reps]
+"""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import torch  # noqa: E402
+
+import bench  # noqa: E402
+import paper_conf_sc_abdelfattahtlad23_b200 as bl  # noqa: E402
+from paper_conf_sc_abdelfattahtlad23_b200 import inputs as I  # noqa: E402
+
+cfg = sys.argv[1] if len(sys.argv) > 1 else "C3"
+reps = int(sys.argv[2]) if len(sys.argv) > 2 else 1
+bpg, n, kl, ku, nrhs, _ = bench.CONFIGS[cfg]
+A0 = torch.from_numpy(I.gen_band(n, n, kl, ku, count=bpg)).cuda()
+B0 = torch.from_numpy(I.gen_rhs(n, nrhs, count=bpg)).cuda()
+A, B = torch.empty_like(A0), torch.empty_like(B0)
+P = torch.zeros((bpg, n), dtype=torch.int32, device="cuda")
+info = torch.zeros(bpg, dtype=torch.int32, device="cuda")
+for _ in range(reps):
+    A.copy_(A0)
+    B.copy_(B0)
+    bl.dgbtrf_strided_batched(n, n, kl, ku, A, P, info)
+    bl.dgbtrs_strided_batched("N", n, kl, ku, A, P, B)
+torch.cuda.synchronize()
+print("ok", cfg, int(info.abs().sum()))
