@@ -35,6 +35,9 @@ namespace {
     X(10, 10)                 \
     X(2, 32)
 
+// trs launch geometry: target resident warps (148 SMs x 8)
+constexpr int64_t kTrsWarpsTarget = 148 * 8;
+
 inline int cuda_ret(cudaError_t e) { return e == cudaSuccess ? 0 : BANDLU_ERR_CUDA + (int)e; }
 
 template <class K>
@@ -102,12 +105,15 @@ int launch_trs_window(int n, int nrhs, AP A, int ldab, PP P, BP B, int ldb, cons
     const int R = nrhs >= 32 ? 32 : pow2_ceil(nrhs);
     const int chunks = (nrhs + 31) / 32;
     auto k = gbtrs_window_kernel<KL, KU, AP, PP, BP>;
-    const size_t sm = C::smem_bytes(R);
-    if (int r = set_smem(k, sm)) return r;
     const int64_t units = (int64_t)batch * chunks;
-    const int gpw = 32 / R;
+    // Each lane runs a long serial chain: spread the units over >= ~8 warps per
+    // SM (all four schedulers busy) before packing more of them into a warp.
+    int gpw = 32 / R;
+    while (gpw > 1 && units < (int64_t)gpw * kTrsWarpsTarget) gpw >>= 1;
+    const size_t sm = C::smem_bytes(R, gpw);
+    if (int r = set_smem(k, sm)) return r;
     const unsigned grid = (unsigned)((units + gpw - 1) / gpw);
-    k<<<grid, 32, sm, st>>>(n, nrhs, A, ldab, P, B, ldb, skip, batch, R, chunks);
+    k<<<grid, 32, sm, st>>>(n, nrhs, A, ldab, P, B, ldb, skip, batch, R, chunks, gpw);
     return cuda_ret(cudaGetLastError());
 }
 

@@ -16,13 +16,15 @@
 //    lanes shares one matrix, 32/R matrices per warp.  Each lane keeps its
 //    sliding RHS window -- KL+1 entries forward, KV+1 backward -- in
 //    registers (slot = row mod window, loop unrolled by the window length),
-//    so the whole serial chain runs in registers.  The row interchange is a
-//    predicated select over the KL window slots.
-//  * Both passes run in ONE kernel; the factor columns and the incoming RHS
-//    entries are staged into a per-warp smem ring by warp-cooperative,
-//    coalesced cp.async (L part only in the forward pass, U part only in the
-//    backward pass, so each factor entry is read from HBM once), NB columns
-//    per stage, double buffered, one __syncwarp per stage.
+//    so the whole serial chain runs in registers; the row interchange is a
+//    predicated select over the window slots.
+//  * Both passes run in ONE kernel.  For every column step the lanes of a
+//    group copy exactly the part of the factor column that pass needs -- L
+//    rows forward, U rows backward, rounded out to 16 B -- with 16-byte
+//    cp.async chunks into an NS-deep per-group smem ring (so each factor
+//    entry is read from HBM once); RHS entries and pivots ride along as
+//    8/4-byte cp.async.  (One bulk/TMA copy per matrix-column was tried: its
+//    uniform operands serialize 32 per-lane copies per step.)
 #pragma once
 #include "common.cuh"
 
@@ -31,112 +33,131 @@ namespace bandlu {
 template <int KL_, int KU_>
 struct TrsWin {
     static constexpr int KL = KL_, KU = KU_, KV = KL + KU;
-    static constexpr int WF = KL + 1, WB = KV + 1;  // forward / backward window lengths
-    static constexpr int NB = 4;                    // columns per stage
-    static constexpr int SLOT = WB > KL ? WB : KL;  // factor doubles per staged column (max of passes)
-    // per-matrix ring: 2 stages x NB x (SLOT factor + 32 max RHS) doubles + 2 x NB ipiv
-    __host__ __device__ static constexpr size_t stage_dbl(int R) { return (size_t)NB * (SLOT + R) + NB / 2 + 1; }
-    __host__ __device__ static constexpr size_t group_dbl(int R) { return (2 * stage_dbl(R)) | 1; }  // odd pitch: conflict-free
-    static constexpr size_t smem_bytes(int R) {
-        return (size_t)(32 / R) * group_dbl(R) * sizeof(double) + (32 / R) * 3 * sizeof(void *);
+    static constexpr int WF = KL + 1, WB = KV + 1;         // forward / backward window lengths
+    static constexpr int NS = 8;                           // ring depth (column steps in flight)
+    static constexpr int FMAX = (KL > WB ? KL : WB) + 2;   // factor doubles per slot (+16 B rounding)
+    static constexpr int SP = (FMAX + 1) & ~1;             // even -> 16 B aligned slots
+    // slot: [SP factor doubles][R rhs doubles][R ipiv ints], padded to an even number of doubles
+    __host__ __device__ static constexpr int slot_dbl(int R) {
+        return ((SP + R + (R + 1) / 2) + 1) & ~1;
     }
+    // group pitch == 2 (mod 4) doubles: lanes of different groups reading the same
+    // slot offset hit different banks (<= 2-way for 64-bit); keeps 16 B alignment
+    __host__ __device__ static constexpr int group_dbl(int R) { return NS * slot_dbl(R) + (6 - (NS * slot_dbl(R)) % 4) % 4; }
+    static constexpr int PAD = (KV + 3) & ~1;  // leading pad: backward reads up to KV doubles before a slot
+    static size_t smem_bytes(int R, int gpw) { return (size_t)(PAD + gpw * group_dbl(R)) * 8; }
 };
 
-// Stage layout for one group (doubles, from the group base):
-//   stage st at st*stage_dbl: [fac: NB*SLOT][rhs: NB*R][piv: NB ints]
 template <int KL, int KU, class AP, class PP, class BP>
 __global__ void __launch_bounds__(32)
     gbtrs_window_kernel(int n, int nrhs, AP A, int ldab, PP P, BP B, int ldb, const int *__restrict__ skip_info,
-                        int batch, int R /* pow2 lanes per matrix */, int chunks /* rhs chunks per matrix */) {
+                        int batch, int R /* pow2 lanes per matrix */, int chunks /* rhs chunks per matrix */,
+                        int gpw /* matrices (groups) per warp, <= 32 / R */) {
     using C = TrsWin<KL, KU>;
-    constexpr int KV = C::KV, WF = C::WF, WB = C::WB, NB = C::NB, SLOT = C::SLOT;
+    constexpr int KV = C::KV, WF = C::WF, WB = C::WB, NS = C::NS, SP = C::SP;
     extern __shared__ __align__(16) double smem[];
     const int lane = (int)lane_id();
-    const int gpw = 32 / R;
     const int g = lane / R, t = lane % R;
     const int64_t unit = (int64_t)blockIdx.x * gpw + g;  // (matrix, rhs chunk)
     const int64_t mat = unit / chunks;
     const int r0 = (int)(unit % chunks) * 32;
-    const int rhs = r0 + t;
-    bool live = unit < (int64_t)batch * chunks;
+    bool live = g < gpw && unit < (int64_t)batch * chunks;
     if (live && skip_info != nullptr && skip_info[mat] != 0) live = false;
-    const bool act = live && rhs < nrhs;  // lane solves (and stores) a column
-    // Dead groups stay in the warp: staging is warp-cooperative.  They compute
-    // on zero-filled data and never touch global memory.
+    const bool act = live && (r0 + t < nrhs);  // lane solves (and stores) a column
     if (__ballot_sync(0xffffffffu, live) == 0u) return;
-    const unsigned wmask = 0xffffffffu;
+    // Dead groups stay (warp-wide barriers); they copy nothing and store nothing.
+    const bool leader = (t == 0);
+
+    const int SD = C::slot_dbl(R), GD = C::group_dbl(R);
+    double *gring = smem + C::PAD + (g < gpw ? g : 0) * GD;
+    const uint32_t gring_s = smem_u32(gring);
+
+    const double *ab = live ? A.get(mat) : nullptr;
+    const int *ipiv = live ? P.get(mat) : nullptr;
+    double *bcol = act ? B.get(mat) + (int64_t)(r0 + t) * ldb : nullptr;  // this lane's RHS column
     const void *dummy = g_dummy;
+    auto slot_rhs_s = [&](int rs) { return gring_s + (uint32_t)((rs * SD + SP + t) * 8); };
+    auto slot_piv_s = [&](int rs) { return gring_s + (uint32_t)((rs * SD + SP + R) * 8 + t * 4); };
 
-    const size_t SD = C::stage_dbl(R), GD = C::group_dbl(R);
-    double **gA = reinterpret_cast<double **>(smem + gpw * GD);
-    int **gP = reinterpret_cast<int **>(gA + gpw);
-    double **gB = reinterpret_cast<double **>(gP + gpw);
-    if (t == 0) {
-        gA[g] = live ? const_cast<double *>(A.get(mat)) : nullptr;
-        gP[g] = live ? const_cast<int *>(P.get(mat)) : nullptr;
-        gB[g] = live ? B.get(mat) + (int64_t)r0 * ldb : nullptr;
-    }
-    __syncwarp();
-    double *gbase = smem + g * GD;
-    double *bcol = act ? gB[g] + (int64_t)t * ldb : nullptr;  // this lane's RHS column
-
-    // --------------------------------------------------------- forward
-    // stage k: columns c in [k*NB, k*NB+NB): L part AB(KV+1+i, c), i < KL
-    // (zero beyond row n-1), ipiv[c], and RHS rows c+KL+1 (zero beyond n-1).
-    auto stage_fwd = [&](int k) {
-        const int c0 = k * NB;
-        const int st = k & 1;
-        if constexpr (KL > 0) {
-            const int EF = NB * KL;
-            for (int e = lane; e < gpw * EF; e += 32) {
-                const int gg = e / EF, rem = e - gg * EF, cc = rem / KL, i = rem - cc * KL;
-                double *dstg = smem + gg * GD + st * SD;
-                const double *a = gA[gg];
-                const int c = c0 + cc;
-                const bool ok = (a != nullptr) && (c + 1 + i < n);
-                cp_async8(smem_u32(dstg + cc * SLOT + i), ok ? a + (int64_t)c * ldab + (KV + 1 + i) : dummy,
-                          ok ? 8u : 0u);
-            }
+    // Global step k: forward steps k < nf (column k), then backward steps
+    // k = nf + kk, kk = 0..n-1 (column n-1-kk).  The factor range of a step:
+    const int nf = KL > 0 ? n : 0;
+    auto fac_range = [&](int k, int64_t &lo, int &cnt) {
+        if (k < nf) {  // L rows KV+1 .. KV+lm of column k
+            const int lm = min(KL, n - 1 - k);
+            lo = (int64_t)k * ldab + KV + 1;
+            cnt = lm > 0 ? lm : 0;
+        } else {  // U rows max(0, KV-j) .. KV of column j
+            const int j = n - 1 - (k - nf);
+            const int r = max(0, KV - j);
+            lo = (int64_t)j * ldab + r;
+            cnt = KV + 1 - r;
         }
-        for (int e = lane; e < gpw * NB * R; e += 32) {
-            const int gg = e / (NB * R), rem = e - gg * (NB * R), rr = rem / NB, cc = rem - rr * NB;
-            double *dstg = smem + gg * GD + st * SD + NB * SLOT;
-            const double *b = gB[gg];
-            const int row = c0 + cc + KL + 1;
-            const bool ok = (b != nullptr) && (row < n) && (r0 + rr < nrhs);
-            cp_async8(smem_u32(dstg + rr * NB + cc), ok ? b + (int64_t)rr * ldb + row : dummy, ok ? 8u : 0u);
-        }
-        for (int e = lane; e < gpw * NB; e += 32) {
-            const int gg = e / NB, cc = e - gg * NB;
-            int *dstg = reinterpret_cast<int *>(smem + gg * GD + st * SD + NB * (SLOT + R));
-            const int *p = gP[gg];
-            const int c = c0 + cc;
-            const bool ok = (p != nullptr) && (c < n);
-            cp_async4(smem_u32(dstg + cc), ok ? (const void *)(p + c) : dummy, ok ? 4u : 0u);
-        }
+    };
+    // 16-byte chunks of the factor range (rounded out), split over the group's lanes
+    auto issue_fac = [&](int k) {
+        if (k >= nf + n || !live) return;
+        int64_t lo;
+        int cnt;
+        fac_range(k, lo, cnt);
+        if (cnt <= 0) return;
+        const uintptr_t a = reinterpret_cast<uintptr_t>(ab + lo);
+        const uintptr_t a0 = a & ~(uintptr_t)15, a1 = (a + (uintptr_t)cnt * 8 + 15) & ~(uintptr_t)15;
+        const int nch = (int)((a1 - a0) >> 4);
+        const uint32_t dst = gring_s + (uint32_t)((k % NS) * SD * 8);
+        for (int q = t; q < nch; q += R) cp_async16(dst + q * 16, reinterpret_cast<const void *>(a0 + q * 16), 16u);
+    };
+    // first needed factor element of step k, inside its slot
+    auto fac_ptr = [&](int k) -> const double * {
+        int64_t lo;
+        int cnt;
+        fac_range(k, lo, cnt);
+        const int delta = live ? (int)((reinterpret_cast<uintptr_t>(ab + lo) >> 3) & 1) : 0;
+        return gring + (k % NS) * SD + delta;
+    };
+    const bool inwarp = g < gpw;  // lanes past the warp's groups own no ring: never copy
+    auto issue_vec_fwd = [&](int k) {  // RHS row k+KL+1 and ipiv[k] for forward step k
+        const int rs = k % NS;
+        if (!inwarp) return;
+        const int row = k + KL + 1;
+        const bool okb = act && row < n;
+        cp_async8(slot_rhs_s(rs), okb ? (const void *)(bcol + row) : dummy, okb ? 8u : 0u);
+        const bool okp = live && k < n;
+        cp_async4(slot_piv_s(rs), okp ? (const void *)(ipiv + k) : dummy, okp ? 4u : 0u);
+        cp_async_commit();
+    };
+    auto issue_vec_bwd = [&](int kk) {  // backward step kk (row j = n-1-kk): RHS row j-KV-1
+        const int rs = (nf + kk) % NS;
+        if (!inwarp) return;
+        const int row = n - 1 - kk - KV - 1;
+        const bool okb = act && row >= 0 && kk < n;
+        cp_async8(slot_rhs_s(rs), okb ? (const void *)(bcol + row) : dummy, okb ? 8u : 0u);
         cp_async_commit();
     };
 
+    // ------------------------------------------------------------ forward
+    // one cp.async group per step: its factor chunks + its RHS entry / pivot
     if constexpr (KL > 0) {
+#pragma unroll 1
+        for (int k = 0; k < NS; ++k) {
+            issue_fac(k);
+            issue_vec_fwd(k);
+        }
         double w[WF];
 #pragma unroll
         for (int i = 0; i < WF; ++i) w[i] = (act && i < n) ? bcol[i] : 0.0;
-        stage_fwd(0);
+#pragma unroll 1
         for (int j0 = 0; j0 < n; j0 += WF) {
 #pragma unroll
             for (int s = 0; s < WF; ++s) {
                 const int j = j0 + s;
                 if (j >= n) break;
-                const int cc = j & (NB - 1);
-                if (cc == 0) {
-                    cp_async_wait<0>();
-                    __syncwarp(wmask);
-                    stage_fwd(j / NB + 1);
-                }
-                const double *sg = gbase + ((j / NB) & 1) * SD;
-                const int *piv = reinterpret_cast<const int *>(sg + NB * (SLOT + R));
+                const int rs = j % NS;
+                cp_async_wait<NS - 1>();
+                __syncwarp();  // chunks copied by the group's other lanes
+                const double *lc = fac_ptr(j);  // lc[i-1] = L(j+i, j); rows >= n: dead slots
                 // interchange B(j) <-> B(l), l in [j, j+KL] (LAPACK never reads ipiv[n-1])
-                const int d = (j < n - 1) ? piv[cc] - 1 - j : 0;
+                const int d = (j < n - 1) ? ld_shared_s32(slot_piv_s(rs)) - 1 - j : 0;
                 double y = w[s];
 #pragma unroll
                 for (int i = 1; i < WF; ++i) {
@@ -147,68 +168,57 @@ __global__ void __launch_bounds__(32)
                 }
                 if (act) bcol[j] = y;
                 if (y != 0.0) {
-                    const double *lc = sg + cc * SLOT;
 #pragma unroll
                     for (int i = 1; i < WF; ++i) w[(s + i) % WF] = __fma_rn(lc[i - 1], -y, w[(s + i) % WF]);
                 }
-                w[s] = sg[NB * SLOT + t * NB + cc];  // RHS row j+KL+1 (0 beyond n)
+                w[s] = ld_shared_f64(slot_rhs_s(rs));  // RHS row j+KL+1 (0 beyond n)
+                __syncwarp();
+                if (j + NS < n) {
+                    issue_fac(j + NS);
+                    issue_vec_fwd(j + NS);
+                } else {
+                    cp_async_commit();
+                }
             }
         }
-        cp_async_wait<0>();
-        __syncwarp(wmask);  // y visible to the backward staging of other lanes
     }
+    cp_async_wait<0>();
+    __threadfence_block();
+    __syncwarp();
 
-    // --------------------------------------------------------- backward
-    // step k handles row j = n-1-k; stage k covers steps [k*NB, k*NB+NB):
-    // U part AB(r, j), r = 0..KV (zero above row 0), RHS rows j-KV-1 (0 if < 0).
-    auto stage_bwd = [&](int k) {
-        const int st = k & 1;
-        const int EU = NB * WB;
-        for (int e = lane; e < gpw * EU; e += 32) {
-            const int gg = e / EU, rem = e - gg * EU, cc = rem / WB, r = rem - cc * WB;
-            double *dstg = smem + gg * GD + st * SD;
-            const double *a = gA[gg];
-            const int j = n - 1 - (k * NB + cc);
-            const bool ok = (a != nullptr) && (j >= 0) && (j - KV + r >= 0);
-            cp_async8(smem_u32(dstg + cc * SLOT + r), ok ? a + (int64_t)j * ldab + r : dummy, ok ? 8u : 0u);
-        }
-        for (int e = lane; e < gpw * NB * R; e += 32) {
-            const int gg = e / (NB * R), rem = e - gg * (NB * R), rr = rem / NB, cc = rem - rr * NB;
-            double *dstg = smem + gg * GD + st * SD + NB * SLOT;
-            const double *b = gB[gg];
-            const int row = n - 1 - (k * NB + cc) - KV - 1;
-            const bool ok = (b != nullptr) && (row >= 0) && (r0 + rr < nrhs);
-            cp_async8(smem_u32(dstg + rr * NB + cc), ok ? b + (int64_t)rr * ldb + row : dummy, ok ? 8u : 0u);
-        }
-        cp_async_commit();
-    };
-
+    // ------------------------------------------------------------ backward
+#pragma unroll 1
+    for (int kk = 0; kk < NS; ++kk) {
+        issue_fac(nf + kk);
+        issue_vec_bwd(kk);
+    }
     double x[WB];
 #pragma unroll
     for (int i = 0; i < WB; ++i) x[i] = (act && n - 1 - i >= 0) ? bcol[n - 1 - i] : 0.0;
-    stage_bwd(0);
-    for (int k0 = 0; k0 < n; k0 += WB) {
+#pragma unroll 1
+    for (int kk0 = 0; kk0 < n; kk0 += WB) {
 #pragma unroll
         for (int s = 0; s < WB; ++s) {
-            const int k = k0 + s;
-            if (k >= n) break;
-            const int j = n - 1 - k;
-            const int cc = k & (NB - 1);
-            if (cc == 0) {
-                cp_async_wait<0>();
-                __syncwarp(wmask);
-                stage_bwd(k / NB + 1);
-            }
-            const double *sg = gbase + ((k / NB) & 1) * SD;
-            const double *uc = sg + cc * SLOT;  // uc[r] = AB(r, j)
+            const int kk = kk0 + s;
+            if (kk >= n) break;
+            const int k = nf + kk, j = n - 1 - kk;
+            const int rs = k % NS;
+            cp_async_wait<NS - 1>();
+            __syncwarp();
+            const double *uc = fac_ptr(k) - max(0, KV - j);  // uc[r] = AB(r, j), r >= KV - j valid
             double xj = x[s];
             if (xj != 0.0) {
                 xj = __ddiv_rn(xj, uc[KV]);
+                // rows j-i < 0 (last KV steps) read the pad / neighbouring slot: they only
+                // feed window slots of rows < 0, which are never stored (dead slots)
 #pragma unroll
                 for (int i = 1; i < WB; ++i) x[(s + i) % WB] = __fma_rn(-xj, uc[KV - i], x[(s + i) % WB]);
             }
             if (act) bcol[j] = xj;
-            x[s] = sg[NB * SLOT + t * NB + cc];  // y(j-KV-1) (0 if < 0)
+            x[s] = ld_shared_f64(slot_rhs_s(rs));  // y(j-KV-1) (0 if < 0)
+            __syncwarp();
+            issue_fac(k + NS);
+            issue_vec_bwd(kk + NS);  // commits the step's group
         }
     }
     cp_async_wait<0>();
