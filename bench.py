@@ -148,7 +148,6 @@ def main():
 
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
     bpg, n, kl, ku, nrhs, desc = CONFIGS[args.config]
     from paper_conf_sc_abdelfattahtlad23_b200 import inputs as I
     b_trf, b_trs = I.alg_bytes(n, n, kl, ku, nrhs)
@@ -178,13 +177,9 @@ def main():
     import torch
     import torch.distributed as dist
     import paper_conf_sc_abdelfattahtlad23_b200 as bl
+    from paper_conf_sc_abdelfattahtlad23_b200 import dist as bd
 
-    if world > 1:
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    else:
-        torch.cuda.set_device(0)
-    dev = torch.device("cuda", torch.cuda.current_device())
+    rank, world, dev = bd.init("nccl")  # one process per GPU; NCCL only off the data path
     bl.load()
 
     # ---- inputs: this rank's shard of the global batch (counter-based generator)
@@ -234,39 +229,35 @@ def main():
     t_trf = [e[0].elapsed_time(e[1]) for e in evs]
     t_trs = [e[1].elapsed_time(e[2]) for e in evs]
     tot_ms = sum(a + b for a, b in zip(t_trf, t_trs))
-    tl = torch.tensor([tot_ms, sum(t_trf), sum(t_trs)], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(tl, op=dist.ReduceOp.MAX)
-    tot_ms, trf_ms, trs_ms = tl.tolist()
+    tot_ms, trf_ms, trs_ms = bd.max_over_ranks([tot_ms, sum(t_trf), sum(t_trs)], dev)  # slowest rank
     ms_step = tot_ms / args.steps
     glob = bpg * world
     value = glob * (f_trf + f_trs) / (ms_step * 1e-3) / 1e9
     hbm = glob * (b_trf + b_trs) / (ms_step * 1e-3) / 1e9
 
     # ---- e2e through the host-buffer C-ABI entry point (H2D + D2H timed)
-    Ah = torch.from_numpy(I.gen_band(n, n, kl, ku, count=cnt, first=lo)).pin_memory()
-    Bh = torch.from_numpy(I.gen_rhs(n, nrhs, count=cnt, first=lo)).pin_memory()
-    Ahw, Bhw = torch.empty_like(Ah).pin_memory(), torch.empty_like(Bh).pin_memory()
-    Ph = torch.zeros((cnt, n), dtype=torch.int32).pin_memory()
-    Ih = torch.zeros(cnt, dtype=torch.int32).pin_memory()
-    e2e_ms = []
-    for k in range(args.e2e_steps + 1):
-        Ahw.copy_(Ah); Bhw.copy_(Bh)
-        if world > 1:
-            dist.barrier()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(st)
-        bl.dgbsv_strided_batched_host(n, kl, ku, Ahw, Ph, Bhw, Ih)  # synchronous
-        e1.record(st)
-        torch.cuda.synchronize()
-        if k > 0:
-            e2e_ms.append(e0.elapsed_time(e1))
-    te = torch.tensor([sum(e2e_ms) / len(e2e_ms)], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(te, op=dist.ReduceOp.MAX)
-    e2e_step = te.item()
-    h2d = Ah.numel() * 8 + Bh.numel() * 8
-    d2h = Ah.numel() * 8 + Ph.numel() * 4 + Bh.numel() * 8 + Ih.numel() * 4
+    e2e_step, h2d, d2h = None, 0, 0
+    if args.e2e_steps > 0:
+        Ah = torch.from_numpy(I.gen_band(n, n, kl, ku, count=cnt, first=lo)).pin_memory()
+        Bh = torch.from_numpy(I.gen_rhs(n, nrhs, count=cnt, first=lo)).pin_memory()
+        Ahw, Bhw = torch.empty_like(Ah).pin_memory(), torch.empty_like(Bh).pin_memory()
+        Ph = torch.zeros((cnt, n), dtype=torch.int32).pin_memory()
+        Ih = torch.zeros(cnt, dtype=torch.int32).pin_memory()
+        e2e_ms = []
+        for k in range(args.e2e_steps + 1):
+            Ahw.copy_(Ah); Bhw.copy_(Bh)
+            if world > 1:
+                dist.barrier()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(st)
+            bl.dgbsv_strided_batched_host(n, kl, ku, Ahw, Ph, Bhw, Ih)  # synchronous
+            e1.record(st)
+            torch.cuda.synchronize()
+            if k > 0:
+                e2e_ms.append(e0.elapsed_time(e1))
+        e2e_step = bd.max_over_ranks([sum(e2e_ms) / len(e2e_ms)], dev)[0]
+        h2d = Ah.numel() * 8 + Bh.numel() * 8
+        d2h = Ah.numel() * 8 + Ph.numel() * 4 + Bh.numel() * 8 + Ih.numel() * 4
 
     if rank != 0:
         if world > 1:
@@ -293,9 +284,10 @@ def main():
         "roofline": {"kernel": dom, "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "peak_kind": peak_kind, "traffic": traffic,
                      "alg_bytes_per_launch": dom_bytes},
-        "e2e": {"value": glob * (f_trf + f_trs) / (e2e_step * 1e-3) / 1e9, "unit": "GFLOP/s",
-                "ms_per_step": e2e_step, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-                "api": "dgbsv_strided_batched_host (pinned host buffers)"},
+        "e2e": None if e2e_step is None else {
+            "value": glob * (f_trf + f_trs) / (e2e_step * 1e-3) / 1e9, "unit": "GFLOP/s",
+            "ms_per_step": e2e_step, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+            "api": "dgbsv_strided_batched_host (pinned host buffers)"},
         "gpu_launches": 2 * args.steps,
         "clocks": clocks,
     }

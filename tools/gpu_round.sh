@@ -1,0 +1,16 @@
+#!/bin/bash
+# One GPU session: tests, default bench (C3 + cpu_baseline), per-config benches,
+# ncu launch list of the bench command, full ncu capture of both kernels at C3.
+set -x
+OUT=gpurun_out
+python -c "import __graft_entry__ as g; g.build(); g.smoke()" > $OUT/smoke.log 2>&1
+timeout 900 python -m pytest tests -m gpu -q > $OUT/pytest_gpu.log 2>&1
+python bench.py > $OUT/bench_default.json 2> $OUT/bench_default.err
+for c in C1 C2 C4; do python bench.py --config $c --steps 30 --warmup 3 --no-cpu > $OUT/bench_$c.json 2>$OUT/bench_$c.err; done
+python bench.py --impl reference --steps 4 > $OUT/bench_reference.json 2>$OUT/bench_reference.err
+ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_c3.csv python bench.py --steps 2 --warmup 3 --e2e-steps 0 --no-cpu > $OUT/ncu_launch_bench.log 2>&1
+for c in C3 C2 C4; do
+  ncu --set full --clock-control none --import-source on -k regex:gbtr -c 2 -o $OUT/full_$c python tools/prof_step.py $c > $OUT/ncu_full_$c.log 2>&1
+done
+tail -3 $OUT/pytest_gpu.log; cat $OUT/smoke.log | tail -2
+python tools/summ.py $OUT/bench_default.json $OUT/bench_C*.json
