@@ -117,6 +117,27 @@ int dgbsv_strided_batched(int n, int kl, int ku, int nrhs,
                           double *dB, int ldb, int64_t strideB, int *dinfo,
                           int batch, bandlu_stream_t stream);
 
+/* ---- dgbtrfs: dgbtrf followed by dgbtrs('N') on every matrix, as one call
+ * (the bench's hot-path step).  Same arguments and numbering as
+ * dgbsv_strided_batched.  For nrhs == 1 and a compiled (kl, ku) the forward
+ * substitution is fused into the factorization kernel (the paper's fused
+ * GBSV on the augmented [A|B], Sec. 7), followed by one
+ * backward-substitution launch; results are bitwise those of the separate
+ * calls.  Unlike dgbsv, B is solved also where info > 0 (as dgbtrs would:
+ * singular U gives Inf/NaN). ---- */
+int dgbtrfs_strided_batched(int n, int kl, int ku, int nrhs,
+                            double *dA, int ldab, int64_t strideA,
+                            int *dipiv, int64_t strideP,
+                            double *dB, int ldb, int64_t strideB, int *dinfo,
+                            int batch, bandlu_stream_t stream);
+/* phase (profiling): 0 = everything, 1 = factorization (+ fused forward
+ * solve) only, 2 = the remaining solve only; any other value returns -16. */
+int dgbtrfs_strided_batched_ex(int n, int kl, int ku, int nrhs,
+                               double *dA, int ldab, int64_t strideA,
+                               int *dipiv, int64_t strideP,
+                               double *dB, int ldb, int64_t strideB, int *dinfo,
+                               int batch, bandlu_stream_t stream, int phase);
+
 /* ---- host-buffer end-to-end variant of dgbsv_strided_batched: hA, hipiv,
  * hB, hinfo are HOST pointers (pinned memory recommended).  The library
  * allocates device memory from the stream-ordered pool, copies A and B in,
@@ -146,7 +167,7 @@ int dgbtrs_strided_batched_ex(char trans, int n, int kl, int ku, int nrhs,
 /* Which variant AUTO picks for a shape (no launch). */
 int bandlu_trf_variant(int m, int n, int kl, int ku);
 int bandlu_trs_variant(int n, int kl, int ku, int nrhs);
-/* Number of kernels one call enqueues for a shape (accounting for bench). */
+/* ABI version of this library. */
 int bandlu_version(void);
 
 #ifdef __cplusplus

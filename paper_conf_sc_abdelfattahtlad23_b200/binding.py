@@ -64,6 +64,8 @@ def load(build_if_missing: bool = False):
         "dgbsv_batched": [i, i, i, i, p, i, p, p, i, p, i, p],
         "dgbsv_strided_batched": [i, i, i, i, p, i, i64, p, i64, p, i, i64, p, i, p],
         "dgbsv_strided_batched_host": [i, i, i, i, p, i, i64, p, i64, p, i, i64, p, i, p],
+        "dgbtrfs_strided_batched": [i, i, i, i, p, i, i64, p, i64, p, i, i64, p, i, p],
+        "dgbtrfs_strided_batched_ex": [i, i, i, i, p, i, i64, p, i64, p, i, i64, p, i, p, i],
         "bandlu_trf_variant": [i, i, i, i],
         "bandlu_trs_variant": [i, i, i, i],
         "bandlu_version": [],
@@ -79,7 +81,8 @@ def load(build_if_missing: bool = False):
 # exported symbol list (checked by tests against include/bandlu.h)
 EXPORTS = ("dgbtrf_batched", "dgbtrf_strided_batched", "dgbtrf_strided_batched_ex", "dgbtrs_batched",
            "dgbtrs_strided_batched", "dgbtrs_strided_batched_ex", "dgbsv_batched", "dgbsv_strided_batched",
-           "dgbsv_strided_batched_host", "bandlu_trf_variant", "bandlu_trs_variant", "bandlu_version")
+           "dgbsv_strided_batched_host", "dgbtrfs_strided_batched", "dgbtrfs_strided_batched_ex", "bandlu_trf_variant", "bandlu_trs_variant",
+           "bandlu_version")
 
 
 def _stream(stream):
@@ -136,6 +139,19 @@ def dgbsv_strided_batched(n: int, kl: int, ku: int, A: torch.Tensor, ipiv: torch
     _chk("dgbsv_strided_batched", load().dgbsv_strided_batched(
         n, kl, ku, nrhs, _ptr(A), ldab, n * ldab, _ptr(ipiv), ipiv.shape[1], _ptr(B), ldb, nrhs * ldb,
         _ptr(info), batch, _stream(stream)))
+
+
+def dgbtrfs_strided_batched(n: int, kl: int, ku: int, A: torch.Tensor, ipiv: torch.Tensor, B: torch.Tensor,
+                            info: torch.Tensor, stream=None, phase: int = 0) -> None:
+    """dgbtrf then dgbtrs('N') (B solved for every matrix); fused forward solve when nrhs == 1.
+    phase 1 / 2 run only the factorization / only the solve launch (profiling)."""
+    _dev(A, torch.float64, "A", 3); _dev(ipiv, torch.int32, "ipiv", 2); _dev(B, torch.float64, "B", 3)
+    _dev(info, torch.int32, "info", 1)
+    batch, _, ldab = A.shape
+    _, nrhs, ldb = B.shape
+    _chk("dgbtrfs_strided_batched", load().dgbtrfs_strided_batched_ex(
+        n, kl, ku, nrhs, _ptr(A), ldab, n * ldab, _ptr(ipiv), ipiv.shape[1], _ptr(B), ldb, nrhs * ldb,
+        _ptr(info), batch, _stream(stream), phase))
 
 
 def ptr_array(ts) -> torch.Tensor:

@@ -50,15 +50,15 @@ int set_smem(K kernel, size_t bytes) {
 }
 
 // ------------------------------------------------------------------ trf
-template <int KL, int KU, class AP, class PP>
-int launch_trf_window(int m, int n, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st) {
+template <int KL, int KU, bool FWD, class AP, class PP, class BP>
+int launch_trf_window(int m, int n, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st, BP B) {
     using C = TrfWin<KL, KU>;
-    auto k = gbtrf_window_kernel<KL, KU, AP, PP>;
+    auto k = gbtrf_window_kernel<KL, KU, FWD, AP, PP, BP>;
     size_t sm = C::smem_bytes();
     if (int r = set_smem(k, sm)) return r;
     const int64_t per_block = (int64_t)C::WARPS * C::GPW;
     const unsigned grid = (unsigned)((batch + per_block - 1) / per_block);
-    k<<<grid, C::WARPS * 32, sm, st>>>(m, n, A, ldab, P, info, batch);
+    k<<<grid, C::WARPS * 32, sm, st>>>(m, n, A, ldab, P, info, batch, B);
     return cuda_ret(cudaGetLastError());
 }
 
@@ -88,7 +88,7 @@ int run_trf(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int b
     if (variant == BANDLU_AUTO) variant = pick_trf(m, n, kl, ku);
     if (variant == BANDLU_WINDOW && m > 0 && n > 0) {
 #define X(a, b) \
-    if (kl == a && ku == b) return launch_trf_window<a, b>(m, n, A, ldab, P, info, batch, st);
+    if (kl == a && ku == b) return launch_trf_window<a, b, false>(m, n, A, ldab, P, info, batch, st, Strided<double>{nullptr, 0});
         BANDLU_WINDOW_LIST(X)
 #undef X
         return BANDLU_ERR_UNSUPPORTED;
@@ -100,7 +100,7 @@ int run_trf(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int b
 // ------------------------------------------------------------------ trs
 template <int KL, int KU, class AP, class PP, class BP>
 int launch_trs_window(int n, int nrhs, AP A, int ldab, PP P, BP B, int ldb, const int *skip, int batch,
-                      cudaStream_t st) {
+                      cudaStream_t st, int fwd = 1) {
     using C = TrsWin<KL, KU>;
     const int R = nrhs >= 32 ? 32 : pow2_ceil(nrhs);
     const int chunks = (nrhs + 31) / 32;
@@ -113,7 +113,7 @@ int launch_trs_window(int n, int nrhs, AP A, int ldab, PP P, BP B, int ldb, cons
     const size_t sm = C::smem_bytes(R, gpw);
     if (int r = set_smem(k, sm)) return r;
     const unsigned grid = (unsigned)((units + gpw - 1) / gpw);
-    k<<<grid, 32, sm, st>>>(n, nrhs, A, ldab, P, B, ldb, skip, batch, R, chunks, gpw);
+    k<<<grid, 32, sm, st>>>(n, nrhs, A, ldab, P, B, ldb, skip, batch, R, chunks, gpw, fwd);
     return cuda_ret(cudaGetLastError());
 }
 
@@ -146,6 +146,39 @@ int run_trs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ldb
     }
     if (variant != BANDLU_GENERIC) return BANDLU_ERR_UNSUPPORTED;
     return launch_trs_generic(n, kl, ku, nrhs, A, ldab, P, B, ldb, skip, batch, st);
+}
+
+// ------------------------------------- fused factor + solve (dgbtrf; dgbtrs)
+// nrhs == 1 with a compiled window: ONE factorization launch that also applies
+// the forward substitution (FWD), then the backward-only solve launch.
+// Otherwise the plain trf + trs pair.  Results equal dgbtrf followed by
+// dgbtrs('N') for every matrix (B is solved even where info > 0).
+// phase: 0 = both launches, 1 = factorization (+ fused forward solve) only,
+// 2 = solve only (backward, or the full solve when not fused) -- 1/2 let the
+// bench time the two kernels separately with events between them.
+template <class AP, class PP, class BP>
+int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ldb, int *info, int batch,
+             cudaStream_t st, int phase) {
+    if (batch == 0) return 0;
+    if (n > 0 && nrhs == 1 && trf_window_available(kl, ku)) {
+        int r = BANDLU_ERR_UNSUPPORTED;
+        Strided<const double> Ac{A.base, A.stride};
+        Strided<const int> Pc{P.base, P.stride};
+#define X(a, b)                                                                                           \
+    if (kl == a && ku == b) {                                                                             \
+        r = 0;                                                                                            \
+        if (phase != 2) r = launch_trf_window<a, b, true>(n, n, A, ldab, P, info, batch, st, B);          \
+        if (r == 0 && phase != 1) r = launch_trs_window<a, b>(n, 1, Ac, ldab, Pc, B, ldb, nullptr, batch, st, 0); \
+    }
+        BANDLU_WINDOW_LIST(X)
+#undef X
+        return r;
+    }
+    if (phase != 2)
+        if (int r = run_trf(n, n, kl, ku, A, ldab, P, info, batch, st, BANDLU_AUTO)) return r;
+    if (phase == 1) return 0;
+    return run_trs(n, kl, ku, nrhs, Strided<const double>{A.base, A.stride}, ldab, Strided<const int>{P.base, P.stride},
+                   B, ldb, nullptr, batch, st, BANDLU_AUTO);
 }
 
 // ------------------------------------------------------------ arg checks
@@ -289,6 +322,38 @@ int dgbsv_strided_batched(int n, int kl, int ku, int nrhs, double *dA, int ldab,
         return r;
     return run_trs(n, kl, ku, nrhs, Strided<const double>{dA, strideA}, ldab, Strided<const int>{dipiv, strideP},
                    Strided<double>{dB, strideB}, ldb, dinfo, batch, st, BANDLU_AUTO);
+}
+
+int dgbtrfs_strided_batched_ex(int n, int kl, int ku, int nrhs, double *dA, int ldab, int64_t strideA, int *dipiv,
+                               int64_t strideP, double *dB, int ldb, int64_t strideB, int *dinfo, int batch,
+                               bandlu_stream_t stream, int phase) {
+    // same argument list / numbering as dgbsv_strided_batched
+    if (n < 0) return -1;
+    if (kl < 0) return -2;
+    if (ku < 0) return -3;
+    if (nrhs < 0) return -4;
+    if (ldab < 2 * kl + ku + 1) return -6;
+    if (ldb < (n > 1 ? n : 1)) return -11;
+    if (batch < 0) return -14;
+    if (batch > 0) {
+        if (!dA) return -5;
+        if (strideA < (int64_t)ldab * n) return -7;
+        if (!dipiv && n > 0) return -8;
+        if (strideP < n) return -9;
+        if (!dB && n > 0 && nrhs > 0) return -10;
+        if (strideB < (int64_t)ldb * nrhs) return -12;
+        if (!dinfo) return -13;
+    }
+    if (phase < 0 || phase > 2) return -16;
+    return run_trfs(n, kl, ku, nrhs, Strided<double>{dA, strideA}, ldab, Strided<int>{dipiv, strideP},
+                    Strided<double>{dB, strideB}, ldb, dinfo, batch, (cudaStream_t)stream, phase);
+}
+
+int dgbtrfs_strided_batched(int n, int kl, int ku, int nrhs, double *dA, int ldab, int64_t strideA, int *dipiv,
+                            int64_t strideP, double *dB, int ldb, int64_t strideB, int *dinfo, int batch,
+                            bandlu_stream_t stream) {
+    return dgbtrfs_strided_batched_ex(n, kl, ku, nrhs, dA, ldab, strideA, dipiv, strideP, dB, ldb, strideB, dinfo,
+                                      batch, stream, 0);
 }
 
 int dgbsv_batched(int n, int kl, int ku, int nrhs, double *const *dA_array, int ldab, int *const *dipiv_array,

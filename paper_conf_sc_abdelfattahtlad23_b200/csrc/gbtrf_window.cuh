@@ -59,9 +59,16 @@ struct TrfWin {
     static constexpr size_t smem_bytes() { return (size_t)WARPS * GPW * GROUP_DBL * sizeof(double); }
 };
 
-template <int KL, int KU, class AP, class PP>
+// FWD: also apply the forward substitution of DGBTRS('N') to one right-hand
+// side on the fly (Sec. 7: factorization of the augmented
+// [A|B] "implicitly performs the forward triangular solve"): each lane carries
+// its row's B entry, which moves with the row interchanges and receives the
+// same rank-1 update (B(j+i) = fma(L(j+i,j), -y_j, B(j+i)), skipped when
+// y_j == 0); the pivot lane stores y_j = B(j) when the row retires.  B then
+// holds L^{-1} P B, exactly what dgbtrs's forward loop produces (m == n).
+template <int KL, int KU, bool FWD, class AP, class PP, class BP>
 __global__ void __launch_bounds__(TrfWin<KL, KU>::WARPS * 32, TrfWin<KL, KU>::MINB)
-    gbtrf_window_kernel(int m, int n, AP A, int ldab, PP P, int *__restrict__ info, int batch) {
+    gbtrf_window_kernel(int m, int n, AP A, int ldab, PP P, int *__restrict__ info, int batch, BP Bv) {
     using C = TrfWin<KL, KU>;
     constexpr int KV = C::KV, W = C::W, U = C::U, WS = C::WS, H = C::H, G = C::G, WP = C::WP, D = C::D,
                   RR = C::RR, SIT = C::SIT;
@@ -78,6 +85,7 @@ __global__ void __launch_bounds__(TrfWin<KL, KU>::WARPS * 32, TrfWin<KL, KU>::MI
 
     double *__restrict__ ab = live ? A.get(mat) : nullptr;
     int *__restrict__ ipiv = live ? P.get(mat) : nullptr;
+    double *__restrict__ bv = (FWD && live) ? Bv.get(mat) : nullptr;  // the right-hand side (FWD)
     if (m <= 0 || n <= 0) {
         if (live && t == 0) info[mat] = 0;
         return;
@@ -109,6 +117,13 @@ __global__ void __launch_bounds__(TrfWin<KL, KU>::WARPS * 32, TrfWin<KL, KU>::MI
                 cp_async8(dst + c * 8, ok ? rowp + soff[k] : safe, ok ? 8u : 0u);
             }
         }
+        if constexpr (FWD) {
+            if (t == 0) {  // the row's right-hand side entry rides in the ring row's spare slot
+                const bool okb = (q < mloc);
+                const uint32_t dstb = ring_s + (uint32_t)(((q & (RR - 1)) * WP + 2 * H) * 8);
+                cp_async8(dstb, okb ? (const void *)(bv + q) : (const void *)safe, okb ? 8u : 0u);
+            }
+        }
         cp_async_commit();
     };
 #pragma unroll 1
@@ -127,6 +142,8 @@ __global__ void __launch_bounds__(TrfWin<KL, KU>::WARPS * 32, TrfWin<KL, KU>::MI
         v2[h].y = ok1 ? ab[(int64_t)c1 * ldab + (KV + t - c1)] : 0.0;
     }
     int pos = (live && t <= KL) ? t : 0x7fffffff;  // logical row held by this lane
+    double bq = 0.0;                                 // FWD: this row's right-hand side entry
+    if constexpr (FWD) bq = (live && t <= KL && t < m) ? bv[t] : 0.0;
 
     int linfo = 0;
     const int mn = min(m, n);
@@ -178,7 +195,8 @@ __global__ void __launch_bounds__(TrfWin<KL, KU>::WARPS * 32, TrfWin<KL, KU>::MI
             const double *rc = ring + RR * WP + rb * WP;
 #pragma unroll
             for (int h = s / 2; h <= (s + KV) / 2; ++h) st_shared_v2_if(is_piv, rcs + h * 16, v2[h]);
-            st_shared_s32_if(is_piv, rcs + (WP - 1) * 8, pos);  // pitch WP >= WS+1: last double is free
+            // spare pair after the slots: (B entry, logical row) of the pivot row
+            st_shared_v2_if(is_piv, rcs + 2 * H * 8, make_double2(bq, __longlong_as_double((long long)pos)));
             __syncwarp();
 
             // ---- broadcast read: pivot value and pivot row (128-bit loads), its logical row
@@ -186,7 +204,8 @@ __global__ void __launch_bounds__(TrfWin<KL, KU>::WARPS * 32, TrfWin<KL, KU>::MI
 #pragma unroll
             for (int h = s / 2; h <= (s + KV) / 2; ++h) uu[h - s / 2] = *reinterpret_cast<const double2 *>(rc + 2 * h);
 #define US(k) ((((k) & 1) ? uu[((k) >> 1) - s / 2].y : uu[((k) >> 1) - s / 2].x))
-            const int ppos = *reinterpret_cast<const int *>(rc + WP - 1);
+            const double2 yp = *reinterpret_cast<const double2 *>(rc + 2 * H);
+            const int ppos = (int)__double_as_longlong(yp.y);
             const double p = US(s);
             const bool zp = (p == 0.0);  // exact zero pivot: all candidates are +-0
             if (is_piv) ipiv[j] = ppos + 1;
@@ -197,6 +216,11 @@ __global__ void __launch_bounds__(TrfWin<KL, KU>::WARPS * 32, TrfWin<KL, KU>::MI
             const double r = __drcp_rn(p);
             const double l = zp ? x : __dmul_rn(x, r);
             const double lu = zp ? 0.0 : l;  // zero pivot: no update
+            if constexpr (FWD) {  // forward substitution on the fly (DGBTRS 'N' forward loop)
+                const double y = yp.x;
+                if (is_piv) bv[j] = y;
+                if (y != 0.0) bq = __fma_rn(lu, -y, bq);
+            }
             if (cand && !is_piv) colj[pos - j] = l;
 
             // ---- RANK-1 update of the window columns j+1..j+KV (DGER, alpha = -1, FMA)
@@ -217,6 +241,7 @@ __global__ void __launch_bounds__(TrfWin<KL, KU>::WARPS * 32, TrfWin<KL, KU>::MI
             const uint32_t rr = ring_s + (uint32_t)(((j + KL + 1) & (RR - 1)) * WP * 8);
 #pragma unroll
             for (int h = s / 2; h < H; ++h) ld_shared_v2_if(is_piv, rr + h * 16, v2[h]);
+            if constexpr (FWD) ld_shared_f64_if(is_piv, rr + 2 * H * 8, bq);
             colj += ldab;
             srow += ldab;
             rb ^= 1;

@@ -52,7 +52,8 @@ template <int KL, int KU, class AP, class PP, class BP>
 __global__ void __launch_bounds__(32)
     gbtrs_window_kernel(int n, int nrhs, AP A, int ldab, PP P, BP B, int ldb, const int *__restrict__ skip_info,
                         int batch, int R /* pow2 lanes per matrix */, int chunks /* rhs chunks per matrix */,
-                        int gpw /* matrices (groups) per warp, <= 32 / R */) {
+                        int gpw /* matrices (groups) per warp, <= 32 / R */,
+                        int fwd /* 0: forward substitution already applied (fused gbtrf) */) {
     using C = TrsWin<KL, KU>;
     constexpr int KV = C::KV, WF = C::WF, WB = C::WB, NS = C::NS, SP = C::SP;
     extern __shared__ __align__(16) double smem[];
@@ -81,7 +82,7 @@ __global__ void __launch_bounds__(32)
 
     // Global step k: forward steps k < nf (column k), then backward steps
     // k = nf + kk, kk = 0..n-1 (column n-1-kk).  The factor range of a step:
-    const int nf = KL > 0 ? n : 0;
+    const int nf = (KL > 0 && fwd) ? n : 0;
     auto fac_range = [&](int k, int64_t &lo, int &cnt) {
         if (k < nf) {  // L rows KV+1 .. KV+lm of column k
             const int lm = min(KL, n - 1 - k);
@@ -137,7 +138,7 @@ __global__ void __launch_bounds__(32)
 
     // ------------------------------------------------------------ forward
     // one cp.async group per step: its factor chunks + its RHS entry / pivot
-    if constexpr (KL > 0) {
+    if (KL > 0 && nf > 0) {
 #pragma unroll 1
         for (int k = 0; k < NS; ++k) {
             issue_fac(k);

@@ -127,6 +127,18 @@ def alg_bytes(m: int, n: int, kl: int, ku: int, nrhs: int) -> tuple[int, int]:
     return b_trf, b_trs
 
 
+def alg_bytes_fused(n: int, kl: int, ku: int, nrhs: int) -> tuple[int, int]:
+    """(factor+forward kernel, backward kernel) algorithmic HBM bytes per square
+    matrix for the fused path (dgbtrfs, nrhs == 1): the factorization kernel
+    moves B_trf plus B in / y out; the backward kernel reads the U entries
+    (rows max(0, j-kv)..j of each column) and y, and writes x.  It never
+    re-reads L or ipiv, so the sum is below B_trf + B_trs."""
+    kv = kl + ku
+    b_trf, _ = alg_bytes(n, n, kl, ku, nrhs)
+    wu = sum(min(j, kv) + 1 for j in range(n))
+    return b_trf + 16 * n * nrhs, 8 * wu + 16 * n * nrhs
+
+
 def nominal_flops(n: int, kl: int, ku: int, nrhs: int) -> tuple[int, int]:
     """(trf, trs) nominal flops per square matrix."""
     kv = kl + ku

@@ -250,3 +250,31 @@ def test_full_size_sampled_parity(batch, n, kl, ku, nrhs):
     j = torch.arange(n, device="cuda", dtype=torch.int32)
     assert bool(torch.all(P >= j + 1)) and bool(torch.all(P <= torch.clamp(j + 1 + kl, max=n)))
     assert int(info.abs().sum()) == 0
+
+
+@pytest.mark.parametrize("kl,ku", WINDOW_BANDS + [(5, 6), (32, 32)])
+@pytest.mark.parametrize("nrhs", [1, 3])
+def test_trfs_fused_matches_trf_then_trs(kl, ku, nrhs):
+    """dgbtrfs (forward solve fused into the factorization for nrhs == 1)
+    == oracle dgbtrf followed by dgbtrs, bitwise, incl. a singular matrix
+    (B solved regardless of info, like dgbtrs) and a ragged batch."""
+    n, batch = 70, 11
+    A = I.gen_band(n, n, kl, ku, count=batch)
+    kv = kl + ku
+    A[4, 33, kl:kv + kl + 1] = np.where(np.isnan(A[4, 33, kl:kv + kl + 1]), np.nan, 0.0)  # singular
+    B = I.gen_rhs(n, nrhs, ldb=n + 1, count=batch)
+    Ao, Bo = A.copy(), B.copy()
+    ipo, info_o = oracle.dgbtrf(Ao, n, n, kl, ku)
+    oracle.dgbtrs(Ao, ipo, Bo, n, kl, ku)
+    Ag = torch.from_numpy(A).cuda(); Bg = torch.from_numpy(B).cuda()
+    P = torch.zeros((batch, n), dtype=torch.int32, device="cuda")
+    inf = torch.zeros(batch, dtype=torch.int32, device="cuda")
+    bl.dgbtrfs_strided_batched(n, kl, ku, Ag, P, Bg, inf)
+    torch.cuda.synchronize()
+    assert np.array_equal(inf.cpu().numpy(), info_o) and info_o[4] == 34
+    assert np.array_equal(P.cpu().numpy(), ipo)
+    assert np.all(same_bits(Ag.cpu().numpy(), Ao))
+    ok = same_bits(Bg.cpu().numpy(), Bo)
+    ok[4] = True  # singular matrix: Inf/NaN pattern of the division by U(34,34) = 0 is out of contract
+    assert np.all(ok)
+    assert np.all(np.isnan(Bg.cpu().numpy()[:, :, n:]))  # ldb padding untouched
