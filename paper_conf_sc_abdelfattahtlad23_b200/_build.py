@@ -7,7 +7,7 @@ import subprocess
 
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
-LIB = os.path.join(PKG, "libbandlu.so")
+LIB = os.environ.get("BANDLU_LIB") or os.path.join(PKG, "libbandlu.so")  # override: experiment builds
 SRC = os.path.join(PKG, "csrc", "bandlu.cu")
 
 NVCC_FLAGS = [

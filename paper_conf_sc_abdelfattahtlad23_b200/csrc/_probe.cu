@@ -1,5 +1,6 @@
-#include "gbtrf_window.cuh"
+#include "gbtrs_window.cuh"
 using namespace bandlu;
 void* probes[] = {
-(void*)&gbtrf_window_kernel<10,10,Strided<double>,Strided<int>>,
+(void*)&gbtrs_window_kernel<10,10,Strided<const double>,Strided<const int>,Strided<double>>,
+(void*)&gbtrs_window_kernel<1,1,Strided<const double>,Strided<const int>,Strided<double>>,
 };

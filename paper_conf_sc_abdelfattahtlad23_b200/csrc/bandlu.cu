@@ -22,6 +22,11 @@ namespace {
 // (KL, KU) pairs compiled into register-resident window kernels (PAPER.md
 // Sec. 8.1 P:897-929 proposes per-(kl, ku) specialisation; we instantiate the
 // bands of the paper's sweeps and of BASELINE.json's configs).
+#ifdef BANDLU_ONLY_C3  // experiment builds: only the (10,10) and (1,1) windows
+#define BANDLU_WINDOW_LIST(X) \
+    X(1, 1)                   \
+    X(10, 10)
+#else
 #define BANDLU_WINDOW_LIST(X) \
     X(0, 0)                   \
     X(0, 3)                   \
@@ -34,6 +39,7 @@ namespace {
     X(10, 7)                  \
     X(10, 10)                 \
     X(2, 32)
+#endif
 
 // trs launch geometry: target resident warps (148 SMs x 8)
 constexpr int64_t kTrsWarpsTarget = 148 * 8;

@@ -38,24 +38,38 @@
 #pragma once
 #include "common.cuh"
 
+// Tuning knobs (compile-time; overridable with -D for experiments)
+#ifndef BANDLU_TRF_U
+#define BANDLU_TRF_U 4
+#endif
+#ifndef BANDLU_TRF_MINB
+#define BANDLU_TRF_MINB 3
+#endif
+#ifndef BANDLU_TRF_WARPS
+#define BANDLU_TRF_WARPS 4
+#endif
+#ifndef BANDLU_TRF_D
+#define BANDLU_TRF_D 8
+#endif
+
 namespace bandlu {
 
 template <int KL_, int KU_>
 struct TrfWin {
     static constexpr int KL = KL_, KU = KU_, KV = KL + KU, W = KV + 1;
-    static constexpr int U = 4;                  // columns per unrolled block (window shift granularity)
+    static constexpr int U = BANDLU_TRF_U;       // columns per unrolled block (window shift granularity)
     static constexpr int WS = W + U;             // register slots: column j0 + r in slot r during a block
     static constexpr int H = (WS + 1) / 2;       // double2 slot pairs
     static constexpr int WP = 2 * H + 2;         // record / ring-row pitch in doubles (16 B rows, +1 free slot)
     static constexpr int G = pow2_ceil(KL + 1);  // lanes per matrix
     static constexpr int GPW = 32 / G;           // matrices per warp
-    static constexpr int D = 8;                  // staging lead (rows)
+    static constexpr int D = BANDLU_TRF_D;       // staging lead (rows)
     static constexpr int RR = 16;                // ring rows (power of 2, > D, multiple of U)
     static constexpr int GROUP_DBL = (RR + 2) * WP;  // ring + 2 pivot-row records (double buffered)
     static constexpr int SIT = (W + G - 1) / G;      // staged elements per lane per row
-    static constexpr int WARPS = 4;
-    // register budget: >= 4 CTAs (16 warps) per SM while the window fits
-    static constexpr int MINB = W <= 24 ? 4 : 2;
+    static constexpr int WARPS = BANDLU_TRF_WARPS;
+    // register budget: >= MINB CTAs per SM while the window fits
+    static constexpr int MINB = W <= 24 ? BANDLU_TRF_MINB : 2;
     static constexpr size_t smem_bytes() { return (size_t)WARPS * GPW * GROUP_DBL * sizeof(double); }
 };
 
@@ -148,6 +162,7 @@ __global__ void __launch_bounds__(TrfWin<KL, KU>::WARPS * 32, TrfWin<KL, KU>::MI
     int linfo = 0;
     const int mn = min(m, n);
     double *colj = live ? ab + KV : nullptr;  // &AB(KV, j)
+    int *ipj = ipiv;                           // &ipiv[j]
     const unsigned gbits = (G == 32) ? 0xffffffffu : ((1u << G) - 1u);
     const unsigned gbase = (unsigned)(g * G);
     int rb = 0;  // pivot-row record buffer of step j (double buffered)
@@ -208,7 +223,7 @@ __global__ void __launch_bounds__(TrfWin<KL, KU>::WARPS * 32, TrfWin<KL, KU>::MI
             const int ppos = (int)__double_as_longlong(yp.y);
             const double p = US(s);
             const bool zp = (p == 0.0);  // exact zero pivot: all candidates are +-0
-            if (is_piv) ipiv[j] = ppos + 1;
+            if (is_piv) *ipj = ppos + 1;
             if (live && zp && linfo == 0) linfo = j + 1;
             if (live && pos == j && !is_piv) pos = ppos;  // interchange = relabel
 
@@ -240,10 +255,11 @@ __global__ void __launch_bounds__(TrfWin<KL, KU>::WARPS * 32, TrfWin<KL, KU>::MI
             if (is_piv) pos = j + KL + 1;
             const uint32_t rr = ring_s + (uint32_t)(((j + KL + 1) & (RR - 1)) * WP * 8);
 #pragma unroll
-            for (int h = s / 2; h < H; ++h) ld_shared_v2_if(is_piv, rr + h * 16, v2[h]);
+            for (int h = (s + 1) / 2; h < H; ++h) ld_shared_v2_if(is_piv, rr + h * 16, v2[h]);  // tail zeros too
             if constexpr (FWD) ld_shared_f64_if(is_piv, rr + 2 * H * 8, bq);
             colj += ldab;
             srow += ldab;
+            ++ipj;
             rb ^= 1;
         }
         // shift the window by U columns: slot r <- slot r+U (U even: whole pairs move)

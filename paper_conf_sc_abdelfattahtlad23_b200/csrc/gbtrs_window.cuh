@@ -95,18 +95,27 @@ __global__ void __launch_bounds__(32)
             cnt = KV + 1 - r;
         }
     };
-    // 16-byte chunks of the factor range (rounded out), split over the group's lanes
+    // 16-byte chunks of the factor range (rounded out).  The copy is split over
+    // CPG = 32/gpw "copy lanes" per group (lane -> group lane/CPG, fixed), so a
+    // warp issues ~nch/CPG chunk copies per lane per step whatever R is.
+    const int CPG = 32 / gpw;
+    const int cg = lane / CPG, cq = lane % CPG;  // copy group / copy lane within it
+    const int64_t cunit = (int64_t)blockIdx.x * gpw + cg;
+    const bool clive = cunit < (int64_t)batch * chunks &&
+                       !(skip_info != nullptr && skip_info[cunit / chunks] != 0);
+    const double *cab = clive ? A.get(cunit / chunks) : nullptr;
+    const uint32_t cring_s = smem_u32(smem + C::PAD + cg * GD);
     auto issue_fac = [&](int k) {
-        if (k >= nf + n || !live) return;
+        if (k >= nf + n || !clive) return;
         int64_t lo;
         int cnt;
         fac_range(k, lo, cnt);
         if (cnt <= 0) return;
-        const uintptr_t a = reinterpret_cast<uintptr_t>(ab + lo);
+        const uintptr_t a = reinterpret_cast<uintptr_t>(cab + lo);
         const uintptr_t a0 = a & ~(uintptr_t)15, a1 = (a + (uintptr_t)cnt * 8 + 15) & ~(uintptr_t)15;
         const int nch = (int)((a1 - a0) >> 4);
-        const uint32_t dst = gring_s + (uint32_t)((k % NS) * SD * 8);
-        for (int q = t; q < nch; q += R) cp_async16(dst + q * 16, reinterpret_cast<const void *>(a0 + q * 16), 16u);
+        const uint32_t dst = cring_s + (uint32_t)((k % NS) * SD * 8);
+        for (int q = cq; q < nch; q += CPG) cp_async16(dst + q * 16, reinterpret_cast<const void *>(a0 + q * 16), 16u);
     };
     // first needed factor element of step k, inside its slot
     auto fac_ptr = [&](int k) -> const double * {

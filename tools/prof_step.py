@@ -24,7 +24,11 @@ info = torch.zeros(bpg, dtype=torch.int32, device="cuda")
 for _ in range(reps):
     A.copy_(A0)
     B.copy_(B0)
-    bl.dgbtrf_strided_batched(n, n, kl, ku, A, P, info)
-    bl.dgbtrs_strided_batched("N", n, kl, ku, A, P, B)
+    if os.environ.get("PROF_SEPARATE"):  # plain dgbtrf + dgbtrs launches
+        bl.dgbtrf_strided_batched(n, n, kl, ku, A, P, info)
+        bl.dgbtrs_strided_batched("N", n, kl, ku, A, P, B)
+    else:  # the bench step: dgbtrfs (fused forward solve when nrhs == 1), two launches
+        bl.dgbtrfs_strided_batched(n, kl, ku, A, P, B, info, phase=1)
+        bl.dgbtrfs_strided_batched(n, kl, ku, A, P, B, info, phase=2)
 torch.cuda.synchronize()
 print("ok", cfg, int(info.abs().sum()))
