@@ -41,6 +41,9 @@ CONFIGS = {  # name: (batch per GPU, n, kl, ku, nrhs, description)
     "C2": (10000, 256, 1, 1, 1, "configs[1]: tridiagonal-like batch=10000, n=256, kl=ku=1, nrhs=1"),
     "C3": (10000, 512, 10, 10, 1, "configs[2]: batch=10000/GPU, n=512, kl=ku=10, nrhs=1 (north_star target)"),
     "C4": (5000, 1024, 2, 32, 16, "configs[3]: batch=5000, n=1024, kl=2, ku=32, nrhs=16"),
+    # application-shaped batches (bands synthetic; the paper gives sizes only)
+    "XGC": (512, 193, 4, 4, 1, "f4 XGC-like: batch=512, n=193 (P:226-227), kl=ku=4, nrhs=1"),
+    "PELE": (10000, 50, 10, 10, 1, "f4 PELE-like: batch=10000, n=50 (P:195-197, 'many <= 50'), kl=ku=10, nrhs=1"),
 }
 
 

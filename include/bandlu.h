@@ -55,8 +55,8 @@
  * -3 kl, -4 ku, -5 nrhs, -7 ldab, -10 ldb; gbsv: -1 n, -2 kl, -3 ku,
  * -4 nrhs, -6 ldab, -9 ldb); batch < 0, a NULL array with batch > 0, or a
  * too-small stride return the position of that argument.  Nothing is
- * enqueued when the return is nonzero.  BANDLU_ERR_UNSUPPORTED: trans other
- * than 'N'/'n' (transposed solve not implemented yet).  BANDLU_ERR_CUDA +
+ * enqueued when the return is nonzero.  BANDLU_ERR_UNSUPPORTED: a forced
+ * variant that is not compiled for the shape.  BANDLU_ERR_CUDA +
  * (cudaError_t) : a launch/runtime error (enqueue failed).
  */
 #ifndef BANDLU_H
@@ -92,8 +92,11 @@ int dgbtrf_strided_batched(int m, int n, int kl, int ku,
                            int *dipiv, int64_t strideP, int *dinfo,
                            int batch, bandlu_stream_t stream);
 
-/* ---- dgbtrs: A X = B with the dgbtrf factors, trans = 'N'.
- * LAPACK DGBTRS semantics: no singularity check (singular U gives Inf/NaN). */
+/* ---- dgbtrs: A X = B (trans 'N'/'n') or A^T X = B (trans 'T'/'t'/'C'/'c',
+ * identical for real data) with the dgbtrf factors (transA).
+ * LAPACK DGBTRS semantics: no singularity check (singular U gives Inf/NaN).
+ * 'T' follows the reference-BLAS operation order of DTBSV('U','T') and
+ * DGEMV('T') (dot products accumulated in increasing index order). */
 int dgbtrs_batched(char trans, int n, int kl, int ku, int nrhs,
                    const double *const *dA_array, int ldab,
                    const int *const *dipiv_array,

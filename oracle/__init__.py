@@ -57,6 +57,8 @@ def _load():
         lib.oracle_dgbtrf_batch.restype = None
         lib.oracle_dgbtrs_n_batch.argtypes = [i, i, i, i, p, i, i64, p, i64, p, i, i64, i, i]
         lib.oracle_dgbtrs_n_batch.restype = None
+        lib.oracle_dgbtrs_t_batch.argtypes = [i, i, i, i, p, i, i64, p, i64, p, i, i64, i, i]
+        lib.oracle_dgbtrs_t_batch.restype = None
         lib.oracle_dgbsv_batch.argtypes = [i, i, i, i, p, i, i64, p, i64, p, i, i64, p, i, i]
         lib.oracle_dgbsv_batch.restype = None
         lib.oracle_max_threads.argtypes = []
@@ -94,13 +96,14 @@ def dgbtrf(A: np.ndarray, m: int, n: int, kl: int, ku: int, nthreads: int = 0,
 
 
 def dgbtrs(A: np.ndarray, ipiv: np.ndarray, B: np.ndarray, n: int, kl: int, ku: int,
-           nthreads: int = 0) -> None:
-    """In-place batched dgbtrs('N') on B [batch, nrhs, ldb] given factors A and ipiv."""
+           nthreads: int = 0, trans: str = "N") -> None:
+    """In-place batched dgbtrs(trans) on B [batch, nrhs, ldb] given factors A and ipiv."""
     _check(A, np.float64, 3, "A"); _check(B, np.float64, 3, "B"); _check(ipiv, np.int32, 2, "ipiv")
     batch, _, ldab = A.shape
     _, nrhs, ldb = B.shape
-    _load().oracle_dgbtrs_n_batch(n, kl, ku, nrhs, _ptr(A), ldab, n * ldab, _ptr(ipiv),
-                                  ipiv.shape[1], _ptr(B), ldb, nrhs * ldb, batch, nthreads)
+    f = _load().oracle_dgbtrs_n_batch if trans.upper() == "N" else _load().oracle_dgbtrs_t_batch
+    f(n, kl, ku, nrhs, _ptr(A), ldab, n * ldab, _ptr(ipiv), ipiv.shape[1], _ptr(B), ldb, nrhs * ldb, batch,
+      nthreads)
 
 
 def dgbsv(A: np.ndarray, B: np.ndarray, n: int, kl: int, ku: int, nthreads: int = 0):

@@ -139,9 +139,22 @@ int pick_trs(int n, int kl, int ku, int nrhs) {
 }
 
 template <class AP, class PP, class BP>
+int launch_trs_t_generic(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ldb, int batch,
+                         cudaStream_t st) {
+    const int64_t threads = (int64_t)batch * nrhs;
+    const unsigned grid = (unsigned)((threads + 127) / 128);
+    gbtrs_t_generic_kernel<AP, PP, BP><<<grid, 128, 0, st>>>(n, kl, ku, nrhs, A, ldab, P, B, ldb, batch);
+    return cuda_ret(cudaGetLastError());
+}
+
+template <class AP, class PP, class BP>
 int run_trs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ldb, const int *skip, int batch,
-            cudaStream_t st, int variant) {
+            cudaStream_t st, int variant, char trans = 'N') {
     if (batch == 0 || n == 0 || nrhs == 0) return 0;
+    if (trans != 'N' && trans != 'n') {  // A^T X = B ('C' == 'T' for real data)
+        if (variant != BANDLU_AUTO && variant != BANDLU_GENERIC) return BANDLU_ERR_UNSUPPORTED;
+        return launch_trs_t_generic(n, kl, ku, nrhs, A, ldab, P, B, ldb, batch, st);
+    }
     if (variant == BANDLU_AUTO) variant = pick_trs(n, kl, ku, nrhs);
     if (variant == BANDLU_WINDOW) {
 #define X(a, b) \
@@ -243,7 +256,6 @@ int check_trs(char trans, int n, int kl, int ku, int nrhs, const void *A, int ld
             if (!B) return -9;
         }
     }
-    if (trans != 'N' && trans != 'n') return BANDLU_ERR_UNSUPPORTED;
     return 0;
 }
 
@@ -283,7 +295,7 @@ int dgbtrs_strided_batched_ex(char trans, int n, int kl, int ku, int nrhs, const
     if (int r = check_trs(trans, n, kl, ku, nrhs, dA, ldab, strideA, dipiv, strideP, dB, ldb, strideB, batch, true))
         return r;
     return run_trs(n, kl, ku, nrhs, Strided<const double>{dA, strideA}, ldab, Strided<const int>{dipiv, strideP},
-                   Strided<double>{dB, strideB}, ldb, nullptr, batch, (cudaStream_t)stream, variant);
+                   Strided<double>{dB, strideB}, ldb, nullptr, batch, (cudaStream_t)stream, variant, trans);
 }
 
 int dgbtrs_strided_batched(char trans, int n, int kl, int ku, int nrhs, const double *dA, int ldab,
@@ -299,7 +311,7 @@ int dgbtrs_batched(char trans, int n, int kl, int ku, int nrhs, const double *co
     if (int r = check_trs(trans, n, kl, ku, nrhs, dA_array, ldab, 0, dipiv_array, 0, dB_array, ldb, 0, batch, false))
         return r;
     return run_trs(n, kl, ku, nrhs, PtrArray<const double>{dA_array}, ldab, PtrArray<const int>{dipiv_array},
-                   PtrArray<double>{dB_array}, ldb, nullptr, batch, (cudaStream_t)stream, BANDLU_AUTO);
+                   PtrArray<double>{dB_array}, ldb, nullptr, batch, (cudaStream_t)stream, BANDLU_AUTO, trans);
 }
 
 int dgbsv_strided_batched(int n, int kl, int ku, int nrhs, double *dA, int ldab, int64_t strideA, int *dipiv,

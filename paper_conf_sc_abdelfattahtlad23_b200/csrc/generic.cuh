@@ -135,4 +135,43 @@ __global__ void __launch_bounds__(128) gbtrs_generic_kernel(int n, int kl, int k
     }
 }
 
+// Transposed solve A^T X = B (LAPACK DGBTRS 'T'/'C' branch; SURVEY 8(f) f2,
+// the transA argument of the paper's dgbtrs_batch).  One thread per
+// (matrix, RHS column), reference-BLAS operation order (one fma per term):
+//   U^T: x_j = (b_j - sum_{i=max(0,j-kv)}^{j-1} U(i,j) x_i) / U(j,j), i ascending
+//   L^T: for j = n-2..0: b_j -= sum_{i=1}^{lm} L(j+i,j) b_{j+i} (dot from 0, i
+//        ascending), then swap b_j <-> b_{ipiv[j]-1}.
+template <class AP, class PP, class BP>
+__global__ void __launch_bounds__(128) gbtrs_t_generic_kernel(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P,
+                                                              BP B, int ldb, int batch) {
+    const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (tid >= (int64_t)batch * nrhs) return;
+    const int mi = (int)(tid / nrhs), r = (int)(tid % nrhs);
+    const double *__restrict__ ab = A.get(mi);
+    const int *__restrict__ ipiv = P.get(mi);
+    double *__restrict__ b = B.get(mi) + (int64_t)r * ldb;
+    const int kv = kl + ku;
+    for (int j = 0; j < n; ++j) {
+        const double *col = ab + (int64_t)j * ldab + kv - j;  // col[i] = AB(kv+i-j, j) = U(i, j)
+        double temp = b[j];
+        for (int i = max(0, j - kv); i <= j - 1; ++i) temp = __fma_rn(-col[i], b[i], temp);
+        b[j] = __ddiv_rn(temp, col[j]);
+    }
+    if (kl > 0) {
+        for (int j = n - 2; j >= 0; --j) {
+            const int lm = min(kl, n - 1 - j);
+            const double *lc = ab + (int64_t)j * ldab + kv;  // lc[i] = L(j+i, j)
+            double temp = 0.0;
+            for (int i = 1; i <= lm; ++i) temp = __fma_rn(b[j + i], lc[i], temp);
+            b[j] = __dsub_rn(b[j], temp);
+            const int l = ipiv[j] - 1;
+            if (l != j) {
+                const double t = b[l];
+                b[l] = b[j];
+                b[j] = t;
+            }
+        }
+    }
+}
+
 }  // namespace bandlu

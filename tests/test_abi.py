@@ -84,7 +84,8 @@ def test_trs_argument_errors(lib):
     assert call(ldb=3) == -12
     assert call(sB=3) == -13
     assert call(batch=-1) == -14
-    assert call(trans=b"T") == 1000  # transposed solve not implemented yet
+    assert call(trans=b"T", batch=0) == 0  # transposed solve supported; batch 0 = quick return
+    assert call(trans=b"c", n=-1) == -2
     g = lib.dgbtrs_batched  # (trans,n,kl,ku,nrhs,A,ldab,P,B,ldb,batch,stream): LAPACK numbering
     assert g(b"N", 4, 1, 1, 1, FAKE, 4, FAKE, FAKE, 3, 1, NULL) == -10
     assert g(b"N", 4, 1, 1, 1, FAKE, 4, NULL, FAKE, 4, 1, NULL) == -8

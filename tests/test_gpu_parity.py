@@ -278,3 +278,39 @@ def test_trfs_fused_matches_trf_then_trs(kl, ku, nrhs):
     ok[4] = True  # singular matrix: Inf/NaN pattern of the division by U(34,34) = 0 is out of contract
     assert np.all(ok)
     assert np.all(np.isnan(Bg.cpu().numpy()[:, :, n:]))  # ldb padding untouched
+
+
+@pytest.mark.parametrize("kl,ku,nrhs", [(2, 3, 2), (10, 10, 1), (1, 1, 3), (0, 4, 1), (4, 0, 2), (2, 32, 16), (33, 20, 1)])
+@pytest.mark.parametrize("trans", ["T", "C"])
+def test_trs_transposed_parity(kl, ku, nrhs, trans):
+    """f2: dgbtrs('T'/'C') on the GPU == oracle (same reference-BLAS order) bitwise."""
+    n, batch = 77, 9
+    A = I.gen_band(n, n, kl, ku, count=batch)
+    ipiv, info = oracle.dgbtrf(A, n, n, kl, ku)
+    B = I.gen_rhs(n, nrhs, ldb=n + 2, count=batch)
+    Bo = B.copy()
+    oracle.dgbtrs(A, ipiv, Bo, n, kl, ku, trans="T")
+    Ag = torch.from_numpy(A).cuda(); Pg = torch.from_numpy(ipiv).cuda(); Bg = torch.from_numpy(B).cuda()
+    bl.dgbtrs_strided_batched(trans, n, kl, ku, Ag, Pg, Bg)
+    torch.cuda.synchronize()
+    assert np.all(same_bits(Bg.cpu().numpy(), Bo))
+
+
+@pytest.mark.parametrize("batch,n,kl,ku", [(512, 193, 4, 4), (2000, 50, 10, 10)])
+def test_application_shaped_workloads(batch, n, kl, ku):
+    """f4: XGC-like (512 x n=193) and PELE-like (n=50)
+    batches through dgbtrfs, every matrix checked against the oracle."""
+    A = I.gen_band(n, n, kl, ku, count=batch)
+    B = I.gen_rhs(n, 1, count=batch)
+    Ao, Bo = A.copy(), B.copy()
+    ipo, info_o = oracle.dgbtrf(Ao, n, n, kl, ku)
+    oracle.dgbtrs(Ao, ipo, Bo, n, kl, ku)
+    Ag = torch.from_numpy(A).cuda(); Bg = torch.from_numpy(B).cuda()
+    P = torch.zeros((batch, n), dtype=torch.int32, device="cuda")
+    inf = torch.zeros(batch, dtype=torch.int32, device="cuda")
+    bl.dgbtrfs_strided_batched(n, kl, ku, Ag, P, Bg, inf)
+    torch.cuda.synchronize()
+    assert np.array_equal(inf.cpu().numpy(), info_o)
+    assert np.array_equal(P.cpu().numpy(), ipo)
+    assert np.all(same_bits(Ag.cpu().numpy(), Ao))
+    assert np.all(same_bits(Bg.cpu().numpy(), Bo))

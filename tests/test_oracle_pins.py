@@ -322,3 +322,47 @@ def test_alg_bytes_match_survey_table():
     assert sum(I.alg_bytes(512, 512, 10, 10, 1)) == 347140
     assert sum(I.alg_bytes(1024, 1024, 2, 32, 16)) == 1149452
     assert I.nominal_flops(512, 10, 10, 1) == (106035, 30702)
+
+
+# ---------------------------------------------------------------- trans = 'T'
+@pytest.mark.parametrize("n,kl,ku,nrhs", [(30, 2, 3, 2), (64, 10, 10, 1), (50, 1, 1, 3), (40, 5, 0, 2),
+                                           (40, 0, 5, 2), (128, 2, 32, 4), (1, 0, 0, 1), (2, 1, 1, 1)])
+def test_trs_transposed_vs_reference_lapack_and_residual(n, kl, ku, nrhs):
+    """f2: dgbtrs('T') solves A^T X = B.  OpenBLAS reorders the dot products,
+    so the pin is (a) normwise agreement with reference LAPACK to 1e-12 and
+    (b) the scaled backward error of A^T x = b <= 10."""
+    A = I.gen_band(n, n, kl, ku, count=3)
+    A0 = A.copy()
+    B = I.gen_rhs(n, nrhs, ldb=n + 2, count=3)
+    B0 = B.copy()
+    ipiv, info = oracle.dgbtrf(A, n, n, kl, ku)
+    oracle.dgbtrs(A, ipiv, B, n, kl, ku, trans="T")
+    for b in range(3):
+        x, inf = L.dgbtrs(A[b].T.copy(order="F"), kl, ku, B0[b].T.copy(order="F"), ipiv[b] - 1, trans=1)
+        X = B[b][:, :n]
+        assert np.abs(x.T[:, :n] - X).max() <= 1e-12 * max(1.0, np.abs(X).max())
+        assert np.all(np.isnan(B[b][:, n:]))
+        D = band_to_dense(A0[b], n, n, kl, ku)
+        assert backward_error(D.T, X.T, B0[b][:, :n].T) <= 10.0
+
+
+def test_trs_transposed_special_cases():
+    # diagonal: x = b / d bitwise
+    n = 20
+    d = I.gen_band(n, n, 0, 0, count=1)
+    B = I.gen_rhs(n, 2, count=1)
+    B0 = B.copy()
+    ipiv, info = oracle.dgbtrf(d, n, n, 0, 0)
+    oracle.dgbtrs(d, ipiv, B, n, 0, 0, trans="T")
+    assert np.array_equal(B[0], B0[0] / d[0, :, 0][None, :])
+    # symmetric tridiag(-1, 2, -1): A^T = A, so 'T' and 'N' solutions agree to rounding
+    n = 50
+    ab = np.full((1, n, 4), np.nan)
+    ab[0, :, 1] = -1.0; ab[0, :, 2] = 2.0; ab[0, :, 3] = -1.0
+    ipiv, info = oracle.dgbtrf(ab, n, n, 1, 1)
+    Bn = np.ones((1, 1, n)); Bt = np.ones((1, 1, n))
+    oracle.dgbtrs(ab, ipiv, Bn, n, 1, 1, trans="N")
+    oracle.dgbtrs(ab, ipiv, Bt, n, 1, 1, trans="T")
+    i = np.arange(1, n + 1)
+    assert np.abs(Bt[0, 0] - i * (n + 1 - i) / 2).max() <= 1e-11
+    assert np.abs(Bt - Bn).max() <= 1e-11
