@@ -61,7 +61,9 @@ struct TrfWin {
     static constexpr int WS = W + U;             // register slots: column j0 + r in slot r during a block
     static constexpr int H = (WS + 1) / 2;       // double2 slot pairs
     static constexpr int WP = 2 * H + 2;         // record / ring-row pitch in doubles (16 B rows, +1 free slot)
-    static constexpr int G = pow2_ceil(KL + 1);  // lanes per matrix
+    // lanes per matrix: pow2 >= KL+1; wide windows use >= 8 so that a warp's
+    // smem rings (and so the resident warps per SM) stay within budget
+    static constexpr int G = pow2_ceil(KL + 1) < (W > 24 ? 8 : 1) ? (W > 24 ? 8 : 1) : pow2_ceil(KL + 1);
     static constexpr int GPW = 32 / G;           // matrices per warp
     static constexpr int D = BANDLU_TRF_D;       // staging lead (rows)
     static constexpr int RR = 16;                // ring rows (power of 2, > D, multiple of U)

@@ -202,13 +202,19 @@ __global__ void __launch_bounds__(32)
         issue_fac(nf + kk);
         issue_vec_bwd(kk);
     }
-    double x[WB];
+    // Backward window: row j-i (i = 0..KV) of step kk = kk0+s sits in slot s+i;
+    // the row entering at step kk (j-WB) goes to slot s+WB.  Blocks of UB steps
+    // are unrolled and the window then shifts down by UB slots (keeps the
+    // kernel small for wide bands; UB = WB for narrow ones = pure rotation).
+    constexpr int UB = WB <= 12 ? WB : 4;
+    constexpr int XS = WB + UB;
+    double x[XS];
 #pragma unroll
-    for (int i = 0; i < WB; ++i) x[i] = (act && n - 1 - i >= 0) ? bcol[n - 1 - i] : 0.0;
+    for (int i = 0; i < XS; ++i) x[i] = (i < WB && act && n - 1 - i >= 0) ? bcol[n - 1 - i] : 0.0;
 #pragma unroll 1
-    for (int kk0 = 0; kk0 < n; kk0 += WB) {
+    for (int kk0 = 0; kk0 < n; kk0 += UB) {
 #pragma unroll
-        for (int s = 0; s < WB; ++s) {
+        for (int s = 0; s < UB; ++s) {
             const int kk = kk0 + s;
             if (kk >= n) break;
             const int k = nf + kk, j = n - 1 - kk;
@@ -222,14 +228,16 @@ __global__ void __launch_bounds__(32)
                 // rows j-i < 0 (last KV steps) read the pad / neighbouring slot: they only
                 // feed window slots of rows < 0, which are never stored (dead slots)
 #pragma unroll
-                for (int i = 1; i < WB; ++i) x[(s + i) % WB] = __fma_rn(-xj, uc[KV - i], x[(s + i) % WB]);
+                for (int i = 1; i < WB; ++i) x[s + i] = __fma_rn(-xj, uc[KV - i], x[s + i]);
             }
             if (act) bcol[j] = xj;
-            x[s] = ld_shared_f64(slot_rhs_s(rs));  // y(j-KV-1) (0 if < 0)
+            x[s + WB] = ld_shared_f64(slot_rhs_s(rs));  // y(j-KV-1) (0 if < 0)
             __syncwarp();
             issue_fac(k + NS);
             issue_vec_bwd(kk + NS);  // commits the step's group
         }
+#pragma unroll
+        for (int i = 0; i < XS; ++i) x[i] = (i + UB < XS) ? x[i + UB] : 0.0;
     }
     cp_async_wait<0>();
 }

@@ -6,7 +6,7 @@ hdr={'trf':'gbtrf_window.cuh','trs':'gbtrs_window.cuh'}[kind]
 lines=['#include "%s"'%hdr,'using namespace bandlu;','void* probes[] = {']
 for kl,ku in pairs:
     if kind=='trf':
-        lines.append('(void*)&gbtrf_window_kernel<%d,%d,Strided<double>,Strided<int>>,'%(kl,ku))
+        lines.append('(void*)&gbtrf_window_kernel<%d,%d,true,Strided<double>,Strided<int>,Strided<double>>,'%(kl,ku))
     else:
         lines.append('(void*)&gbtrs_window_kernel<%d,%d,Strided<const double>,Strided<const int>,Strided<double>>,'%(kl,ku))
 lines.append('};')
