@@ -14,27 +14,30 @@
 //    warp (per-warp instruction cost is shared by all of them).
 //  * Row-owner mapping: each of the KL+1 active lanes holds ONE row of the
 //    active window -- the W = KL+KU+1 values at columns j..j+KV -- in
-//    registers, column c in slot c mod W, slots paired into double2 so rows
-//    move to/from shared memory with 128-bit accesses.  The column loop is
-//    unrolled W times: sliding the window never moves a register.
+//    registers.  Columns are processed in blocks of U = 4: during a block,
+//    column j0+r sits in register slot r (slots paired into double2 so rows
+//    move to/from shared memory with 128-bit accesses); after the block the
+//    slots shift down by U (register moves), which keeps the unrolled code
+//    small enough for the instruction cache.
 //  * Row interchanges are relabelings: a lane carries the logical position of
 //    its row.  LAPACK swaps only columns j..ju; beyond ju both rows hold
 //    structural zeros, so swapping whole rows is identical.
-//  * IAMAX: butterfly max of the high word of the |x| bit pattern + ballot;
+//  * IAMAX: warp REDUX max of the high word of the |x| bit pattern + ballot;
 //    exact slow path (low word, then smallest logical row) only when the
 //    high words tie (zero pivots, exact ties) -- first-max semantics (Q2).
-//  * The pivot row is broadcast to its group with width-G shuffles (the
-//    shuffle path runs beside the shared-memory pipe, which the row staging
-//    and the U store use); every lane then applies the rank-1 update with
-//    FP64 FMAs in registers.  The pivot lane also drops its row (= U row j)
-//    into a double-buffered smem record that the group stores to HBM one
-//    step later.  Multipliers are stored by their owning lanes.
-//  * Input rows are gathered one row per step by cp.async (LDGSTS,
-//    L1-allocating, zero-fill outside the matrix) into a 16-row smem ring in
-//    slot order, D = 8 rows ahead; the lane freed by the pivot row reloads
-//    its registers from it with 128-bit loads.  Fill rows (input) are never
-//    read; every input element is read from HBM once, every output element
-//    written once.
+//  * The pivot lane drops its row (= U row j) and (B entry, logical row)
+//    into an smem record; the group reads it back with 128-bit broadcast
+//    loads and every lane applies the rank-1 update with FP64 FMAs in
+//    registers.  Multipliers (band column j below the diagonal, contiguous)
+//    are stored by their owning lanes each step.
+//  * Global traffic moves in blocks of U rows: in band storage U consecutive
+//    rows of one column are U contiguous doubles, so U lanes move one 32-byte
+//    chunk.  Input rows j0+KL+1+D .. +U are gathered by cp.async (LDGSTS,
+//    zero-fill outside the matrix) into an smem ring, D rows ahead; the lane
+//    freed by a pivot row reloads its registers from the ring with 128-bit
+//    loads.  The block's U pivot records are stored as U rows at block end.
+//    Fill rows (input) are never read; every input element is read from HBM
+//    once, every output element written once.
 #pragma once
 #include "common.cuh"
 
@@ -49,7 +52,10 @@
 #define BANDLU_TRF_WARPS 4
 #endif
 #ifndef BANDLU_TRF_D
-#define BANDLU_TRF_D 8
+#define BANDLU_TRF_D 8  // staging lead in rows for groups of >= 8 lanes (4 below)
+#endif
+#ifndef BANDLU_TRF_SHFL_BCAST
+#define BANDLU_TRF_SHFL_BCAST 0
 #endif
 
 namespace bandlu {
@@ -60,18 +66,29 @@ struct TrfWin {
     static constexpr int U = BANDLU_TRF_U;       // columns per unrolled block (window shift granularity)
     static constexpr int WS = W + U;             // register slots: column j0 + r in slot r during a block
     static constexpr int H = (WS + 1) / 2;       // double2 slot pairs
-    static constexpr int WP = 2 * H + 2;         // record / ring-row pitch in doubles (16 B rows, +1 free slot)
+    // Ring rows and pivot-row records are indexed by block slot (16-byte slot
+    // pairs), then a spare pair at RP: (B entry) in ring rows, (B entry,
+    // logical row) in records.  Pitch WP == 2 (mod 4) doubles.
+    static constexpr int RP = 2 * H + ((2 * H + 2) % 4 == 2 ? 0 : 2);
+    static constexpr int WP = RP + 2;
     // lanes per matrix: pow2 >= KL+1; wide windows use >= 8 so that a warp's
     // smem rings (and so the resident warps per SM) stay within budget
     static constexpr int G = pow2_ceil(KL + 1) < (W > 24 ? 8 : 1) ? (W > 24 ? 8 : 1) : pow2_ceil(KL + 1);
     static constexpr int GPW = 32 / G;           // matrices per warp
-    static constexpr int D = BANDLU_TRF_D;       // staging lead (rows)
-    static constexpr int RR = 16;                // ring rows (power of 2, > D, multiple of U)
-    static constexpr int GROUP_DBL = (RR + 2) * WP;  // ring + 2 pivot-row records (double buffered)
-    static constexpr int SIT = (W + G - 1) / G;      // staged elements per lane per row
-    static constexpr int WARPS = BANDLU_TRF_WARPS;
+    static constexpr int D = G >= 8 ? BANDLU_TRF_D : U;  // staging lead (rows, multiple of U)
+    static constexpr int DB = D / U;             // staging lead in blocks
+    static constexpr int RR = pow2_ceil((DB + 1) * U);  // ring rows (power of 2, multiple of U)
+    static constexpr int NREC = U;               // pivot-row records: this block's U rows
+    static constexpr int GROUP_DBL = (RR + NREC) * WP;  // input-row ring + pivot-row records
+    // Block transfers (U rows at a time): in band storage U consecutive rows of
+    // one column are U contiguous doubles, so U lanes move one column chunk.
+    static constexpr int BK = W + U - 1;         // columns touched by U consecutive rows
+    static constexpr int BIT = (BK * U + G - 1) / G;  // block elements per lane
+    // warps per CTA: up to BANDLU_TRF_WARPS while a CTA's rings fit ~76 KB (3 CTAs/SM)
+    static constexpr int WARPS_FIT = (76 * 1024) / (GPW * GROUP_DBL * 8);
+    static constexpr int WARPS = WARPS_FIT < 1 ? 1 : (WARPS_FIT < BANDLU_TRF_WARPS ? WARPS_FIT : BANDLU_TRF_WARPS);
     // register budget: >= MINB CTAs per SM while the window fits
-    static constexpr int MINB = W <= 24 ? BANDLU_TRF_MINB : 2;
+    static constexpr int MINB = (W <= 24 ? BANDLU_TRF_MINB * 4 : 8) / WARPS;  // (12 or 8 resident warps)
     static constexpr size_t smem_bytes() { return (size_t)WARPS * GPW * GROUP_DBL * sizeof(double); }
 };
 
@@ -86,9 +103,9 @@ template <int KL, int KU, bool FWD, class AP, class PP, class BP>
 __global__ void __launch_bounds__(TrfWin<KL, KU>::WARPS * 32, TrfWin<KL, KU>::MINB)
     gbtrf_window_kernel(int m, int n, AP A, int ldab, PP P, int *__restrict__ info, int batch, BP Bv) {
     using C = TrfWin<KL, KU>;
-    constexpr int KV = C::KV, W = C::W, U = C::U, WS = C::WS, H = C::H, G = C::G, WP = C::WP, D = C::D,
-                  RR = C::RR, SIT = C::SIT;
-    static_assert(U % 2 == 0 && RR % U == 0, "block geometry");
+    constexpr int KV = C::KV, W = C::W, U = C::U, WS = C::WS, H = C::H, G = C::G, WP = C::WP, RP = C::RP, D = C::D,
+                  RR = C::RR, BK = C::BK, BIT = C::BIT;
+    static_assert(U % 2 == 0 && RR % U == 0 && D % U == 0 && (U & (U - 1)) == 0, "block geometry");
     extern __shared__ __align__(16) double smem[];
 
     const int lane = (int)lane_id(), wib = (int)(threadIdx.x >> 5);
@@ -112,39 +129,61 @@ __global__ void __launch_bounds__(TrfWin<KL, KU>::WARPS * 32, TrfWin<KL, KU>::MI
     const uint32_t rec_s = ring_s + RR * WP * 8;
     const double *safe = live ? ab : g_dummy;  // zero-fill copies never read it
 
-    // Ring row of input row q (loaded at step j = q-KL-1, block offset o = j % U)
+    // Ring row of input row q (needed at step q-KL-1, block offset o = (q-KL-1) % U)
     // holds A(q, q-KL+c) at position o+1+c, zeros elsewhere, so one 128-bit
     // load per slot pair drops it into the window registers.  o is fixed per
     // ring row (RR % U == 0), so the zero positions are zeroed once here.
     for (int i = t; i < RR * WP; i += G) ring[i] = 0.0;
     __syncwarp();
 
-    // ---- staging: lane t copies c = t + k*G (element at AB(KV+KL-c, q-KL+c))
-    int soff[SIT];
+    // ---- block element e = t + k*G of this lane: row offset bs = e % U, column
+    // offset bk = e / U.  Rows qb..qb+U-1 (qb = first row of a block, qb-KL-1 a
+    // multiple of U) span columns qb-KL .. qb-KL+BK-1; A(qb+bs, qb-KL+bk) sits at
+    // AB(KV+KL+bs-bk, qb-KL+bk) and (c = bk-bs in 0..KV) at ring position 1+bk.
+    // U rows of the previous block: record bs holds U row j0+bs at slots
+    // bs..bs+KV; U(j0+bs, j0+bk) goes to AB(KV+bs-bk, j0+bk).  Both are U
+    // contiguous doubles per column: U lanes, one 32-byte chunk.
+    // element offset from &AB(0, first column): bk*(ldab-1) + bs
+    const int bo0 = (t / U) * (ldab - 1) + (t % U), bstep = (G / U) * (ldab - 1);
+    auto boff = [&](int k) -> int {
+        if constexpr (G % U == 0) return bo0 + k * bstep;  // bs fixed per lane
+        const int e = t + k * G;
+        return (e / U) * (ldab - 1) + (e % U);
+    };
+    unsigned bmask = 0;  // bit k: element k lies inside the band row (0 <= bk-bs <= KV)
 #pragma unroll
-    for (int k = 0; k < SIT; ++k) soff[k] = (t + k * G) * (ldab - 1) + (KV + KL);
-    auto stage_row = [&](int q, const double *rowp) {
-        const uint32_t dst = ring_s + (uint32_t)(((q & (RR - 1)) * WP + 1 + ((q - KL - 1) & (U - 1))) * 8);
+    for (int k = 0; k < BIT; ++k) {
+        const int e = t + k * G, bs = e % U, bk = e / U;
+        if (bk < BK && bk - bs >= 0 && bk - bs <= KV) bmask |= 1u << k;
+    }
+    // rows qb..qb+U-1 -> ring (cp.async, zero-fill outside the matrix);
+    // colq = &AB(0, qb-KL).  One commit group per block.
+    auto stage_block = [&](int qb, const double *colq) {
 #pragma unroll
-        for (int k = 0; k < SIT; ++k) {
-            const int c = t + k * G;
-            if (c < W) {
-                const bool ok = (q < mloc) && (q - KL + c < n);
-                cp_async8(dst + c * 8, ok ? rowp + soff[k] : safe, ok ? 8u : 0u);
+        for (int k = 0; k < BIT; ++k) {
+            const int e = t + k * G, bs = e % U, bk = e / U;
+            if (bmask >> k & 1u) {
+                const int q = qb + bs;
+                const bool ok = (q < mloc) && (qb - KL + bk < n);
+                const uint32_t dst = ring_s + (uint32_t)(((q & (RR - 1)) * WP + 1 + bk) * 8);
+                cp_async8(dst, ok ? colq + boff(k) + (KV + KL) : safe, ok ? 8u : 0u);
             }
         }
         if constexpr (FWD) {
-            if (t == 0) {  // the row's right-hand side entry rides in the ring row's spare slot
+#pragma unroll
+            for (int i = t; i < U; i += G) {  // the row's right-hand side entry rides in the ring row's spare slot
+                const int q = qb + i;
                 const bool okb = (q < mloc);
-                const uint32_t dstb = ring_s + (uint32_t)(((q & (RR - 1)) * WP + 2 * H) * 8);
+                const uint32_t dstb = ring_s + (uint32_t)(((q & (RR - 1)) * WP + RP) * 8);
                 cp_async8(dstb, okb ? (const void *)(bv + q) : (const void *)safe, okb ? 8u : 0u);
             }
         }
         cp_async_commit();
     };
 #pragma unroll 1
-    for (int d = 0; d < D; ++d) stage_row(KL + 1 + d, live ? ab + (int64_t)(1 + d) * ldab : g_dummy);
-    const double *srow = live ? ab + (int64_t)(1 + D) * ldab : g_dummy;  // &A(q-KL, .) of the row staged next
+    for (int d = 0; d < C::DB; ++d)
+        stage_block(KL + 1 + d * U, live ? ab + (int64_t)(1 + d * U) * ldab : g_dummy);
+    const double *scol = live ? ab + (int64_t)(1 + D) * ldab : g_dummy;  // &AB(0, qb-KL) of the block staged next
 
     // ---- window registers (slot pairs): slot r = column j0 + r; rows 0..KL first
     double2 v2[H];
@@ -164,17 +203,20 @@ __global__ void __launch_bounds__(TrfWin<KL, KU>::WARPS * 32, TrfWin<KL, KU>::MI
     int linfo = 0;
     const int mn = min(m, n);
     double *colj = live ? ab + KV : nullptr;  // &AB(KV, j)
+    double *colb = live ? ab : nullptr;       // &AB(0, j0)
     int *ipj = ipiv;                           // &ipiv[j]
     const unsigned gbits = (G == 32) ? 0xffffffffu : ((1u << G) - 1u);
     const unsigned gbase = (unsigned)(g * G);
-    int rb = 0;  // pivot-row record buffer of step j (double buffered)
 #pragma unroll 1
     for (int j0 = 0; j0 < mn; j0 += U) {
+        cp_async_wait<C::DB - 1>();  // rows j0+KL+1 .. j0+KL+U landed (this lane's part; the
+                                     // __syncwarp below publishes them to the pivot lanes)
+        stage_block(j0 + KL + 1 + D, scol);
+        scol += (int64_t)U * ldab;
 #pragma unroll
         for (int s = 0; s < U; ++s) {  // column j = j0 + s sits in slot s
             const int j = j0 + s;
             if (j >= mn) break;
-            cp_async_wait<D - 1>();  // row j+KL+1 landed (this lane's part)
 
             // ---- IAMAX over the candidates (logical rows j..min(j+KL, m-1))
             const double x = VS(s);
@@ -208,20 +250,32 @@ __global__ void __launch_bounds__(TrfWin<KL, KU>::WARPS * 32, TrfWin<KL, KU>::MI
             const bool is_piv = (t == __ffs(gb) - 1);  // dead groups: gb = 0, nobody
 
             // ---- pivot row (U row j: slots s..s+KV) + its logical row -> smem record, 128-bit
-            const uint32_t rcs = rec_s + (uint32_t)(rb * WP * 8);
-            const double *rc = ring + RR * WP + rb * WP;
+            const uint32_t rcs = rec_s + (uint32_t)(s * WP * 8);
+            const double *rc = reinterpret_cast<const double *>(ring) + (rcs - ring_s) / 8;
 #pragma unroll
             for (int h = s / 2; h <= (s + KV) / 2; ++h) st_shared_v2_if(is_piv, rcs + h * 16, v2[h]);
             // spare pair after the slots: (B entry, logical row) of the pivot row
-            st_shared_v2_if(is_piv, rcs + 2 * H * 8, make_double2(bq, __longlong_as_double((long long)pos)));
+            st_shared_v2_if(is_piv, rcs + RP * 8, make_double2(bq, __longlong_as_double((long long)pos)));
             __syncwarp();
 
-            // ---- broadcast read: pivot value and pivot row (128-bit loads), its logical row
+            // ---- broadcast read: pivot value and pivot row, its logical row
+#if BANDLU_TRF_SHFL_BCAST
+            // width-G shuffles from the pivot lane (runs beside the smem pipe)
+            const int src = (int)gbase + __ffs(gb | (gb == 0u)) - 1;
+            double uu[W];
+#pragma unroll
+            for (int k = 0; k <= KV; ++k) uu[k] = __shfl_sync(0xffffffffu, VS(s + k), src);
+#define US(k) (uu[(k) - s])
+            double2 yp;
+            yp.x = __shfl_sync(0xffffffffu, bq, src);
+            yp.y = __longlong_as_double((long long)__shfl_sync(0xffffffffu, pos, src));
+#else
             double2 uu[KV / 2 + 2];
 #pragma unroll
             for (int h = s / 2; h <= (s + KV) / 2; ++h) uu[h - s / 2] = *reinterpret_cast<const double2 *>(rc + 2 * h);
 #define US(k) ((((k) & 1) ? uu[((k) >> 1) - s / 2].y : uu[((k) >> 1) - s / 2].x))
-            const double2 yp = *reinterpret_cast<const double2 *>(rc + 2 * H);
+            const double2 yp = *reinterpret_cast<const double2 *>(rc + RP);
+#endif
             const int ppos = (int)__double_as_longlong(yp.y);
             const double p = US(s);
             const bool zp = (p == 0.0);  // exact zero pivot: all candidates are +-0
@@ -245,25 +299,25 @@ __global__ void __launch_bounds__(TrfWin<KL, KU>::WARPS * 32, TrfWin<KL, KU>::MI
             for (int k = s + 1; k <= s + KV; ++k) VS(k) = __fma_rn(lu, -US(k), VS(k));
 #undef US
 
-            // ---- U row j -> HBM: U(j, j+c) = record[s + c] at AB(KV-c, j+c)
-#pragma unroll
-            for (int k = 0; k < SIT; ++k) {
-                const int c = t + k * G;
-                if (live && c < W && j + c < n) colj[(int64_t)c * (ldab - 1)] = rc[s + c];
-            }
-            stage_row(j + KL + 1 + D, srow);
-
             // ---- slide: the pivot lane takes row j+KL+1 (ring row pre-positioned at slots s+1..s+W)
             if (is_piv) pos = j + KL + 1;
             const uint32_t rr = ring_s + (uint32_t)(((j + KL + 1) & (RR - 1)) * WP * 8);
 #pragma unroll
             for (int h = (s + 1) / 2; h < H; ++h) ld_shared_v2_if(is_piv, rr + h * 16, v2[h]);  // tail zeros too
-            if constexpr (FWD) ld_shared_f64_if(is_piv, rr + 2 * H * 8, bq);
+            if constexpr (FWD) ld_shared_f64_if(is_piv, rr + RP * 8, bq);
             colj += ldab;
-            srow += ldab;
             ++ipj;
-            rb ^= 1;
         }
+        // ---- U rows j0 .. j0+U-1 (this block's pivot rows) -> HBM, 32-byte column chunks
+        __syncwarp();
+#pragma unroll
+        for (int k = 0; k < BIT; ++k) {
+            const int e = t + k * G, bs = e % U, bk = e / U;
+            if (live && (bmask >> k & 1u) && j0 + bs < mn && j0 + bk < n)
+                colb[boff(k) + KV] = ld_shared_f64(rec_s + (uint32_t)((bs * WP + bk) * 8));
+        }
+        colb += (int64_t)U * ldab;
+        __syncwarp();  // records are rewritten by the next block's pivot lanes
         // shift the window by U columns: slot r <- slot r+U (U even: whole pairs move)
 #pragma unroll
         for (int h = 0; h < H; ++h) {
@@ -276,6 +330,7 @@ __global__ void __launch_bounds__(TrfWin<KL, KU>::WARPS * 32, TrfWin<KL, KU>::MI
         }
     }
     cp_async_wait<0>();
+    __syncwarp();
 #undef VS
     if (!live) return;
 
