@@ -52,7 +52,10 @@
 #define BANDLU_TRF_WARPS 4
 #endif
 #ifndef BANDLU_TRF_D
-#define BANDLU_TRF_D 8  // staging lead in rows for groups of >= 8 lanes (4 below)
+#define BANDLU_TRF_D 4  // staging lead in rows (multiple of U; 8 measured slower on C3)
+#endif
+#ifndef BANDLU_TRF_WP16
+#define BANDLU_TRF_WP16 1
 #endif
 #ifndef BANDLU_TRF_SHFL_BCAST
 #define BANDLU_TRF_SHFL_BCAST 0
@@ -69,13 +72,18 @@ struct TrfWin {
     // Ring rows and pivot-row records are indexed by block slot (16-byte slot
     // pairs), then a spare pair at RP: (B entry) in ring rows, (B entry,
     // logical row) in records.  Pitch WP == 2 (mod 4) doubles.
-    static constexpr int RP = 2 * H + ((2 * H + 2) % 4 == 2 ? 0 : 2);
-    static constexpr int WP = RP + 2;
+    // Wide rows (>= 8-lane groups): WP == 4 (mod 16), so the U x U chunk
+    // patterns of the block transfers (row offset bs, column offset bk ->
+    // bs*WP + bk) hit 16 distinct 8-byte banks; short rows: WP == 2 (mod 4)
+    // (smaller rings, measured better there).
+    static constexpr int WP = (BANDLU_TRF_WP16 && pow2_ceil(KL + 1) >= 8) ? ((2 * H + 2 + 11) / 16) * 16 + 4
+                                                                          : 2 * H + 2 + ((2 * H + 2) % 4 == 2 ? 0 : 2);
+    static constexpr int RP = WP - 2;
     // lanes per matrix: pow2 >= KL+1; wide windows use >= 8 so that a warp's
     // smem rings (and so the resident warps per SM) stay within budget
     static constexpr int G = pow2_ceil(KL + 1) < (W > 24 ? 8 : 1) ? (W > 24 ? 8 : 1) : pow2_ceil(KL + 1);
     static constexpr int GPW = 32 / G;           // matrices per warp
-    static constexpr int D = G >= 8 ? BANDLU_TRF_D : U;  // staging lead (rows, multiple of U)
+    static constexpr int D = BANDLU_TRF_D;       // staging lead (rows, multiple of U)
     static constexpr int DB = D / U;             // staging lead in blocks
     static constexpr int RR = pow2_ceil((DB + 1) * U);  // ring rows (power of 2, multiple of U)
     static constexpr int NREC = U;               // pivot-row records: this block's U rows
