@@ -79,7 +79,10 @@ typedef struct CUstream_st *bandlu_stream_t;
 enum bandlu_variant {
     BANDLU_AUTO = 0,
     BANDLU_GENERIC = 1, /* warp-per-matrix in-place kernel, any m, n, kl, ku (safeguard) */
-    BANDLU_WINDOW = 2   /* register-resident sliding window, compiled (kl, ku) only (Sec. 5.3 / 8.1) */
+    BANDLU_WINDOW = 2,  /* register-resident sliding window, compiled (kl, ku) only (Sec. 5.3 / 8.1) */
+    BANDLU_TC = 3       /* dgbtrf only, opt-in: window in FP64 tensor-core (DMMA) fragments, compiled
+                           (kl, ku) with kl+1 <= 16 (bandlu_tc_available); same LAPACK operation
+                           sequence, bitwise equal results */
 };
 
 /* ---- dgbtrf: band LU with partial pivoting ---- */
@@ -170,6 +173,10 @@ int dgbtrs_strided_batched_ex(char trans, int n, int kl, int ku, int nrhs,
 /* Which variant AUTO picks for a shape (no launch). */
 int bandlu_trf_variant(int m, int n, int kl, int ku);
 int bandlu_trs_variant(int n, int kl, int ku, int nrhs);
+/* 1 if a tensor-core (BANDLU_TC) factorization kernel is compiled for (kl, ku),
+ * else 0 (no launch).  BANDLU_TC is never chosen by AUTO; force it with
+ * dgbtrf_strided_batched_ex. */
+int bandlu_tc_available(int kl, int ku);
 /* ABI version of this library. */
 int bandlu_version(void);
 

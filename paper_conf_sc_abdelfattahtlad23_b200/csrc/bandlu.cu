@@ -11,6 +11,7 @@
 
 #include "../../include/bandlu.h"
 #include "common.cuh"
+#include "gbtrf_tc.cuh"
 #include "gbtrf_window.cuh"
 #include "gbtrs_window.cuh"
 #include "generic.cuh"
@@ -26,6 +27,7 @@ namespace {
 #define BANDLU_WINDOW_LIST(X) \
     X(1, 1)                   \
     X(10, 10)
+#define BANDLU_TC_LIST(X) X(10, 10)
 #else
 #define BANDLU_WINDOW_LIST(X) \
     X(0, 0)                   \
@@ -39,6 +41,13 @@ namespace {
     X(10, 7)                  \
     X(10, 10)                 \
     X(2, 32)
+// (KL, KU) pairs also compiled as tensor-core (DMMA) factorization kernels
+// (kl+1 <= 16; preferred by AUTO where compiled).
+#ifdef BANDLU_NO_TC
+#define BANDLU_TC_LIST(X)
+#else
+#define BANDLU_TC_LIST(X) X(10, 10)
+#endif
 #endif
 
 // trs launch geometry: target resident warps (148 SMs x 8)
@@ -83,15 +92,43 @@ bool trf_window_available(int kl, int ku) {
     return false;
 }
 
+bool trf_tc_available(int kl, int ku) {
+#define X(a, b) \
+    if (kl == a && ku == b) return true;
+    BANDLU_TC_LIST(X)
+#undef X
+    return false;
+}
+
 int pick_trf(int m, int n, int kl, int ku) {
     if (m <= 0 || n <= 0) return BANDLU_GENERIC;
+    // BANDLU_TC is opt-in: measured slower than the row-owner window at C3
+    // (1.54 vs 1.10 ms), so AUTO never picks it.
     return trf_window_available(kl, ku) ? BANDLU_WINDOW : BANDLU_GENERIC;
+}
+
+template <int KL, int KU, bool FWD, class AP, class PP, class BP>
+int launch_trf_tc(int m, int n, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st, BP B) {
+    using C = TrfTc<KL, KU>;
+    auto k = gbtrf_tc_kernel<KL, KU, FWD, AP, PP, BP>;
+    size_t sm = C::smem_bytes();
+    if (int r = set_smem(k, sm)) return r;
+    const unsigned grid = (unsigned)((batch + C::WARPS - 1) / C::WARPS);
+    k<<<grid, C::WARPS * 32, sm, st>>>(m, n, A, ldab, P, info, batch, B);
+    return cuda_ret(cudaGetLastError());
 }
 
 template <class AP, class PP>
 int run_trf(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st, int variant) {
     if (batch == 0) return 0;
     if (variant == BANDLU_AUTO) variant = pick_trf(m, n, kl, ku);
+    if (variant == BANDLU_TC && m > 0 && n > 0) {
+#define X(a, b) \
+    if (kl == a && ku == b) return launch_trf_tc<a, b, false>(m, n, A, ldab, P, info, batch, st, Strided<double>{nullptr, 0});
+        BANDLU_TC_LIST(X)
+#undef X
+        return BANDLU_ERR_UNSUPPORTED;
+    }
     if (variant == BANDLU_WINDOW && m > 0 && n > 0) {
 #define X(a, b) \
     if (kl == a && ku == b) return launch_trf_window<a, b, false>(m, n, A, ldab, P, info, batch, st, Strided<double>{nullptr, 0});
@@ -99,7 +136,7 @@ int run_trf(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int b
 #undef X
         return BANDLU_ERR_UNSUPPORTED;
     }
-    if (variant != BANDLU_GENERIC && variant != BANDLU_WINDOW) return BANDLU_ERR_UNSUPPORTED;
+    if (variant != BANDLU_GENERIC && variant != BANDLU_WINDOW && variant != BANDLU_TC) return BANDLU_ERR_UNSUPPORTED;
     return launch_trf_generic(m, n, kl, ku, A, ldab, P, info, batch, st);
 }
 
@@ -267,6 +304,7 @@ extern "C" {
 int bandlu_version(void) { return 1; }
 
 int bandlu_trf_variant(int m, int n, int kl, int ku) { return pick_trf(m, n, kl, ku); }
+int bandlu_tc_available(int kl, int ku) { return trf_tc_available(kl, ku) ? 1 : 0; }
 int bandlu_trs_variant(int n, int kl, int ku, int nrhs) { return pick_trs(n, kl, ku, nrhs); }
 
 int dgbtrf_strided_batched_ex(int m, int n, int kl, int ku, double *dA, int ldab, int64_t strideA, int *dipiv,

@@ -91,6 +91,11 @@ __device__ __forceinline__ void st_shared_v2_if(bool p, uint32_t a, double2 v) {
                  "r"(a), "d"(v.x), "d"(v.y)
                  : "memory");
 }
+__device__ __forceinline__ double2 ld_shared_v2(uint32_t a) {
+    double2 v;
+    asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];\n" : "=d"(v.x), "=d"(v.y) : "r"(a) : "memory");
+    return v;
+}
 __device__ __forceinline__ void ld_shared_v2_if(bool p, uint32_t a, double2 &v) {
     asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %2, 0;\n\t@q ld.shared.v2.f64 {%0, %1}, [%3];\n\t}\n"
                  : "+d"(v.x), "+d"(v.y)

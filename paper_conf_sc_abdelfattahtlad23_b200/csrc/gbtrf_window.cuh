@@ -57,9 +57,6 @@
 #ifndef BANDLU_TRF_WP16
 #define BANDLU_TRF_WP16 1
 #endif
-#ifndef BANDLU_TRF_SHFL_BCAST
-#define BANDLU_TRF_SHFL_BCAST 0
-#endif
 
 namespace bandlu {
 
@@ -267,23 +264,11 @@ __global__ void __launch_bounds__(TrfWin<KL, KU>::WARPS * 32, TrfWin<KL, KU>::MI
             __syncwarp();
 
             // ---- broadcast read: pivot value and pivot row, its logical row
-#if BANDLU_TRF_SHFL_BCAST
-            // width-G shuffles from the pivot lane (runs beside the smem pipe)
-            const int src = (int)gbase + __ffs(gb | (gb == 0u)) - 1;
-            double uu[W];
-#pragma unroll
-            for (int k = 0; k <= KV; ++k) uu[k] = __shfl_sync(0xffffffffu, VS(s + k), src);
-#define US(k) (uu[(k) - s])
-            double2 yp;
-            yp.x = __shfl_sync(0xffffffffu, bq, src);
-            yp.y = __longlong_as_double((long long)__shfl_sync(0xffffffffu, pos, src));
-#else
             double2 uu[KV / 2 + 2];
 #pragma unroll
             for (int h = s / 2; h <= (s + KV) / 2; ++h) uu[h - s / 2] = *reinterpret_cast<const double2 *>(rc + 2 * h);
 #define US(k) ((((k) & 1) ? uu[((k) >> 1) - s / 2].y : uu[((k) >> 1) - s / 2].x))
             const double2 yp = *reinterpret_cast<const double2 *>(rc + RP);
-#endif
             const int ppos = (int)__double_as_longlong(yp.y);
             const double p = US(s);
             const bool zp = (p == 0.0);  // exact zero pivot: all candidates are +-0

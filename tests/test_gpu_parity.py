@@ -34,6 +34,15 @@ def _gpu_trf(A_np, m, n, kl, ku, variant=bl.AUTO):
     return A.cpu().numpy(), ipiv.cpu().numpy()[:, :min(m, n)], info.cpu().numpy()
 
 
+def trf_variants(kl, ku):
+    """Forced factorization variants to cross-check: the safeguard, the row-owner
+    window, and the tensor-core (DMMA) kernel where it is compiled for (kl, ku)."""
+    v = [bl.WINDOW, bl.GENERIC]
+    if bl.tc_available(kl, ku):
+        v.append(bl.TC)
+    return v
+
+
 def _check_trf(m, n, kl, ku, batch, variant, ldab=None, first=0, A_in=None):
     A0 = I.gen_band(m, n, kl, ku, ldab=ldab, count=batch, first=first) if A_in is None else A_in
     Ao = A0.copy()
@@ -47,9 +56,11 @@ def _check_trf(m, n, kl, ku, batch, variant, ldab=None, first=0, A_in=None):
 
 
 @pytest.mark.parametrize("kl,ku", WINDOW_BANDS)
-@pytest.mark.parametrize("variant", [bl.WINDOW, bl.GENERIC])
+@pytest.mark.parametrize("variant", [bl.WINDOW, bl.GENERIC, bl.TC])
 @pytest.mark.parametrize("n", [1, 2, 7, 37, 100])
 def test_trf_parity_small(kl, ku, variant, n):
+    if variant not in trf_variants(kl, ku):
+        pytest.skip("no tensor-core kernel compiled for this band")
     # ragged batch (not a multiple of matrices per warp / block)
     _check_trf(n, n, kl, ku, batch=37, variant=variant)
 
@@ -58,7 +69,7 @@ def test_trf_parity_small(kl, ku, variant, n):
 @pytest.mark.parametrize("mn", [(30, 20), (20, 30), (5, 40), (40, 5), (1, 9), (9, 1)])
 def test_trf_parity_rectangular(kl, ku, mn):
     m, n = mn
-    for variant in (bl.WINDOW, bl.GENERIC):
+    for variant in trf_variants(kl, ku):
         _check_trf(m, n, kl, ku, batch=9, variant=variant)
 
 
@@ -71,7 +82,7 @@ def test_trf_parity_generic_any_band(kl, ku):
 @pytest.mark.parametrize("kl,ku", [(1, 1), (10, 10), (2, 32)])
 def test_trf_parity_padded_ldab(kl, ku):
     ldab = 2 * kl + ku + 1 + 3  # extra NaN rows at the bottom stay untouched
-    for variant in (bl.WINDOW, bl.GENERIC):
+    for variant in trf_variants(kl, ku):
         _check_trf(70, 70, kl, ku, batch=5, variant=variant, ldab=ldab)
 
 
@@ -84,7 +95,7 @@ def test_trf_parity_planted_zero_pivots(kl, ku):
         col = A[b, z - 1, kl:kv + kl + 1]
         A[b, z - 1, kl:kv + kl + 1] = np.where(np.isnan(col), np.nan, 0.0)
     A[5, 10, kl:kv + kl + 1] = np.where(np.isnan(A[5, 10, kl:kv + kl + 1]), np.nan, 0.0)  # two zeros
-    for variant in (bl.WINDOW, bl.GENERIC):
+    for variant in trf_variants(kl, ku):
         Ao, ipo, info = _check_trf(n, n, kl, ku, 6, variant, A_in=A.copy())
         assert list(info) == [1, 2, 30, 59, 60, 11]
 
@@ -96,7 +107,7 @@ def test_trf_parity_exact_ties(kl, ku):
     n = 64
     A = I.gen_band(n, n, kl, ku, count=16)
     A = np.where(np.isnan(A), np.nan, np.sign(A) * np.ceil(np.abs(A) * 2.0))  # values in {+-1, +-2}
-    for variant in (bl.WINDOW, bl.GENERIC):
+    for variant in trf_variants(kl, ku):
         _check_trf(n, n, kl, ku, 16, variant, A_in=A.copy())
 
 
