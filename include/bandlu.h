@@ -145,11 +145,13 @@ int dgbtrfs_strided_batched_ex(int n, int kl, int ku, int nrhs,
                                int batch, bandlu_stream_t stream, int phase);
 
 /* ---- host-buffer end-to-end variant of dgbsv_strided_batched: hA, hipiv,
- * hB, hinfo are HOST pointers (pinned memory recommended).  The library
- * allocates device memory from the stream-ordered pool, copies A and B in,
- * factors and solves, copies A (factors), ipiv, B (solution) and info back,
- * and synchronizes `stream` before returning.  Work is pipelined over batch
- * chunks so copies overlap the kernels.  Returns as above, or
+ * hB, hinfo are HOST pointers (pinned memory recommended).  The library keeps
+ * three streams and three ~64 MB device staging buffers per process (created
+ * on first use on the current device, grown on demand, never freed), copies
+ * A and B in, factors and solves, copies A (factors), ipiv, B (solution) and
+ * info back, and synchronizes `stream` before returning.  Batch chunks are
+ * pipelined so host->device copies, kernels and device->host copies overlap.
+ * Calls are serialized by a process-wide lock.  Returns as above, or
  * BANDLU_ERR_CUDA + err on an allocation / copy failure. */
 int dgbsv_strided_batched_host(int n, int kl, int ku, int nrhs,
                                double *hA, int ldab, int64_t strideA,

@@ -443,6 +443,52 @@ int dgbsv_batched(int n, int kl, int ku, int nrhs, double *const *dA_array, int 
 // Pipelined over batch chunks on two internal streams: H2D(A_c, B_c) ->
 // gbtrf -> gbtrs -> D2H(A_c, ipiv_c, B_c, info_c); chunk c+1's copies overlap
 // chunk c's kernels (separate copy engines for each direction).
+namespace {
+// Device-side state of the host-buffer entry point, kept across calls so an
+// e2e call pays no allocation: NS streams and one staging buffer per stream
+// (grown on demand, on the device of the call).
+struct HostPipe {
+    static constexpr int NS = 3;
+    std::mutex mu;
+    int dev = -1;
+    cudaStream_t s[NS] = {};
+    cudaEvent_t done[NS] = {};
+    cudaEvent_t start = nullptr;
+    void *buf[NS] = {};
+    size_t cap = 0;
+    cudaError_t prepare(size_t need) {
+        int d = 0;
+        cudaError_t e = cudaGetDevice(&d);
+        if (e != cudaSuccess) return e;
+        if (d != dev) {  // first call, or another device: (re)create streams and events
+            for (int i = 0; i < NS; ++i) buf[i] = nullptr;  // buffers of another device are abandoned
+            cap = 0;
+            for (int i = 0; i < NS; ++i) {
+                if ((e = cudaStreamCreateWithFlags(&s[i], cudaStreamNonBlocking)) != cudaSuccess) return e;
+                if ((e = cudaEventCreateWithFlags(&done[i], cudaEventDisableTiming)) != cudaSuccess) return e;
+            }
+            if ((e = cudaEventCreateWithFlags(&start, cudaEventDisableTiming)) != cudaSuccess) return e;
+            dev = d;
+        }
+        if (need > cap) {
+            for (int i = 0; i < NS; ++i) {
+                if (buf[i]) {
+                    cudaStreamSynchronize(s[i]);
+                    cudaFree(buf[i]);
+                    buf[i] = nullptr;
+                }
+            }
+            cap = 0;
+            for (int i = 0; i < NS; ++i)
+                if ((e = cudaMalloc(&buf[i], need)) != cudaSuccess) return e;
+            cap = need;
+        }
+        return cudaSuccess;
+    }
+};
+HostPipe g_pipe;
+}  // namespace
+
 extern "C" int dgbsv_strided_batched_host(int n, int kl, int ku, int nrhs, double *hA, int ldab, int64_t strideA,
                                           int *hipiv, int64_t strideP, double *hB, int ldb, int64_t strideB,
                                           int *hinfo, int batch, bandlu_stream_t stream) {
@@ -464,67 +510,48 @@ extern "C" int dgbsv_strided_batched_host(int n, int kl, int ku, int nrhs, doubl
 
     cudaStream_t user = (cudaStream_t)stream;
     const int64_t bytes_per = strideA * 8 + strideB * 8 + strideP * 4 + 4;
-    int64_t ch = (int64_t)((256ll << 20) / (bytes_per > 0 ? bytes_per : 1));  // ~256 MB per chunk
-    ch = ch < 1 ? 1 : ch;
-    if (ch > (batch + 3) / 4) ch = (batch + 3) / 4;  // at least ~4 chunks for overlap
-    if (ch < 1) ch = 1;
+    // ~64 MB chunks over NS = 3 streams: H2D of chunk c+1, the kernels of chunk c
+    // and D2H of chunk c-1 overlap (PCIe copy engines run both directions at once)
+    int64_t ch = (int64_t)((64ll << 20) / (bytes_per > 0 ? bytes_per : 1));
+    ch = ch < 1 ? 1 : (ch > batch ? batch : ch);
     const int nchunks = (int)((batch + ch - 1) / ch);
+    const size_t offB = (size_t)ch * strideA * 8, offP = offB + (((size_t)ch * strideB * 8 + 15) & ~(size_t)15);
+    const size_t offI = offP + (((size_t)ch * strideP * 4 + 15) & ~(size_t)15);
+    const size_t need = offI + (size_t)ch * 4 + 16;
 
-    cudaError_t e;
-    cudaStream_t s[2] = {nullptr, nullptr};
-    cudaEvent_t ev0 = nullptr, ev[2] = {nullptr, nullptr};
-    double *dA[2] = {nullptr, nullptr}, *dB[2] = {nullptr, nullptr};
-    int *dP[2] = {nullptr, nullptr}, *dI[2] = {nullptr, nullptr};
+    std::lock_guard<std::mutex> lock(g_pipe.mu);
     int ret = 0;
-    auto fail = [&](cudaError_t err) { if (!ret) ret = cuda_ret(err); };
-    for (int i = 0; i < 2; ++i) {
-        if ((e = cudaStreamCreateWithFlags(&s[i], cudaStreamNonBlocking)) != cudaSuccess) fail(e);
-        if ((e = cudaEventCreateWithFlags(&ev[i], cudaEventDisableTiming)) != cudaSuccess) fail(e);
-    }
-    if ((e = cudaEventCreateWithFlags(&ev0, cudaEventDisableTiming)) != cudaSuccess) fail(e);
-    if (!ret) {
-        cudaEventRecord(ev0, user);
-        for (int i = 0; i < 2 && !ret; ++i) {
-            cudaStreamWaitEvent(s[i], ev0, 0);
-            if ((e = cudaMallocAsync((void **)&dA[i], (size_t)(ch * strideA * 8), s[i])) != cudaSuccess) fail(e);
-            if ((e = cudaMallocAsync((void **)&dB[i], (size_t)(ch * strideB * 8 + 8), s[i])) != cudaSuccess) fail(e);
-            if ((e = cudaMallocAsync((void **)&dP[i], (size_t)(ch * strideP * 4 + 4), s[i])) != cudaSuccess) fail(e);
-            if ((e = cudaMallocAsync((void **)&dI[i], (size_t)(ch * 4), s[i])) != cudaSuccess) fail(e);
-        }
-    }
-    for (int c = 0; c < nchunks && !ret; ++c) {
-        const int i = c & 1;
+    cudaError_t e;
+    if ((e = g_pipe.prepare(need)) != cudaSuccess) return cuda_ret(e);
+    cudaEvent_t ev0 = g_pipe.start;
+    cudaEventRecord(ev0, user);
+    for (int i = 0; i < HostPipe::NS; ++i) cudaStreamWaitEvent(g_pipe.s[i], ev0, 0);
+    for (int c = 0; c < nchunks; ++c) {
+        const int i = c % HostPipe::NS;
+        cudaStream_t si = g_pipe.s[i];
+        char *base = (char *)g_pipe.buf[i];
+        double *dA = (double *)base, *dB = (double *)(base + offB);
+        int *dP = (int *)(base + offP), *dI = (int *)(base + offI);
         const int64_t b0 = (int64_t)c * ch;
         const int cb = (int)((batch - b0) < ch ? (batch - b0) : ch);
         const size_t aN = (size_t)((cb - 1) * strideA + (int64_t)ldab * n);
         const size_t bN = (size_t)((cb - 1) * strideB + (int64_t)ldb * nrhs);
         const size_t pN = (size_t)((cb - 1) * strideP + n);
-        cudaMemcpyAsync(dA[i], hA + b0 * strideA, aN * 8, cudaMemcpyHostToDevice, s[i]);
-        if (bN) cudaMemcpyAsync(dB[i], hB + b0 * strideB, bN * 8, cudaMemcpyHostToDevice, s[i]);
-        int r = dgbsv_strided_batched(n, kl, ku, nrhs, dA[i], ldab, strideA, dP[i], strideP, dB[i], ldb, strideB,
-                                      dI[i], cb, (bandlu_stream_t)s[i]);
+        cudaMemcpyAsync(dA, hA + b0 * strideA, aN * 8, cudaMemcpyHostToDevice, si);
+        if (bN) cudaMemcpyAsync(dB, hB + b0 * strideB, bN * 8, cudaMemcpyHostToDevice, si);
+        int r = dgbsv_strided_batched(n, kl, ku, nrhs, dA, ldab, strideA, dP, strideP, dB, ldb, strideB, dI, cb,
+                                      (bandlu_stream_t)si);
         if (r) { ret = r; break; }
-        cudaMemcpyAsync(hA + b0 * strideA, dA[i], aN * 8, cudaMemcpyDeviceToHost, s[i]);
-        if (pN && n > 0) cudaMemcpyAsync(hipiv + b0 * strideP, dP[i], pN * 4, cudaMemcpyDeviceToHost, s[i]);
-        if (bN) cudaMemcpyAsync(hB + b0 * strideB, dB[i], bN * 8, cudaMemcpyDeviceToHost, s[i]);
-        cudaMemcpyAsync(hinfo + b0, dI[i], (size_t)cb * 4, cudaMemcpyDeviceToHost, s[i]);
-        if ((e = cudaGetLastError()) != cudaSuccess) fail(e);
+        cudaMemcpyAsync(hA + b0 * strideA, dA, aN * 8, cudaMemcpyDeviceToHost, si);
+        if (pN && n > 0) cudaMemcpyAsync(hipiv + b0 * strideP, dP, pN * 4, cudaMemcpyDeviceToHost, si);
+        if (bN) cudaMemcpyAsync(hB + b0 * strideB, dB, bN * 8, cudaMemcpyDeviceToHost, si);
+        cudaMemcpyAsync(hinfo + b0, dI, (size_t)cb * 4, cudaMemcpyDeviceToHost, si);
+        if ((e = cudaGetLastError()) != cudaSuccess) { ret = cuda_ret(e); break; }
     }
-    for (int i = 0; i < 2; ++i) {
-        if (s[i]) {
-            if (dA[i]) cudaFreeAsync(dA[i], s[i]);
-            if (dB[i]) cudaFreeAsync(dB[i], s[i]);
-            if (dP[i]) cudaFreeAsync(dP[i], s[i]);
-            if (dI[i]) cudaFreeAsync(dI[i], s[i]);
-            cudaEventRecord(ev[i], s[i]);
-            cudaStreamWaitEvent(user, ev[i], 0);
-        }
+    for (int i = 0; i < HostPipe::NS; ++i) {
+        cudaEventRecord(g_pipe.done[i], g_pipe.s[i]);
+        cudaStreamWaitEvent(user, g_pipe.done[i], 0);
     }
-    if ((e = cudaStreamSynchronize(user)) != cudaSuccess) fail(e);
-    for (int i = 0; i < 2; ++i) {
-        if (s[i]) cudaStreamDestroy(s[i]);
-        if (ev[i]) cudaEventDestroy(ev[i]);
-    }
-    if (ev0) cudaEventDestroy(ev0);
+    if ((e = cudaStreamSynchronize(user)) != cudaSuccess && !ret) ret = cuda_ret(e);
     return ret;
 }

@@ -210,6 +210,27 @@ def test_host_buffer_gbsv_matches_oracle():
     assert np.array_equal(P.numpy(), ipo) and np.array_equal(inf.numpy(), info_o)
 
 
+def test_host_buffer_gbsv_many_chunks():
+    """The host entry point pipelines ~64 MB chunks over 3 reused device buffers:
+    4+ chunks with a ragged tail, a singular matrix (B untouched), nrhs 2 with
+    padded ldb, then a second call on a larger problem (buffers grow)."""
+    for n, kl, ku, nrhs, batch in [(32, 1, 1, 2, 130000), (40, 3, 2, 1, 200000)]:
+        ldb = n + 3
+        A = I.gen_band(n, n, kl, ku, count=batch)
+        B = I.gen_rhs(n, nrhs, ldb=ldb, count=batch)
+        kv = kl + ku
+        A[7, 5, kl:kv + kl + 1] = np.where(np.isnan(A[7, 5, kl:kv + kl + 1]), np.nan, 0.0)  # singular
+        Ao, Bo = A.copy(), B.copy()
+        ipo, info_o = oracle.dgbsv(Ao, Bo, n, kl, ku)
+        assert info_o[7] == 6
+        At = torch.from_numpy(A).pin_memory(); Bt = torch.from_numpy(B).pin_memory()
+        P = torch.zeros((batch, n), dtype=torch.int32).pin_memory()
+        inf = torch.zeros(batch, dtype=torch.int32).pin_memory()
+        bl.dgbsv_strided_batched_host(n, kl, ku, At, P, Bt, inf)
+        assert np.array_equal(inf.numpy(), info_o) and np.array_equal(P.numpy(), ipo)
+        assert np.all(same_bits(At.numpy(), Ao)) and np.all(same_bits(Bt.numpy(), Bo))
+
+
 def test_quick_returns_write_info():
     A = torch.zeros((5, 3, 4), dtype=torch.float64, device="cuda")
     ipiv = torch.zeros((5, 1), dtype=torch.int32, device="cuda")

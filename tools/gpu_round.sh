@@ -6,7 +6,7 @@ OUT=gpurun_out
 python -c "import __graft_entry__ as g; g.build(); g.smoke()" > $OUT/smoke.log 2>&1
 timeout 900 python -m pytest tests -m gpu -q > $OUT/pytest_gpu.log 2>&1
 python bench.py > $OUT/bench_default.json 2> $OUT/bench_default.err
-for c in C1 C2 C4; do python bench.py --config $c --steps 30 --warmup 3 --no-cpu > $OUT/bench_$c.json 2>$OUT/bench_$c.err; done
+for c in C1 C2 C4 XGC PELE; do python bench.py --config $c --steps 30 --warmup 3 --no-cpu > $OUT/bench_$c.json 2>$OUT/bench_$c.err; done
 python bench.py --impl reference --steps 4 > $OUT/bench_reference.json 2>$OUT/bench_reference.err
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_c3.csv python bench.py --steps 2 --warmup 3 --e2e-steps 0 --no-cpu > $OUT/ncu_launch_bench.log 2>&1
 for c in C3 C2 C4; do
