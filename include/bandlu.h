@@ -80,9 +80,12 @@ enum bandlu_variant {
     BANDLU_AUTO = 0,
     BANDLU_GENERIC = 1, /* warp-per-matrix in-place kernel, any m, n, kl, ku (safeguard) */
     BANDLU_WINDOW = 2,  /* register-resident sliding window, compiled (kl, ku) only (Sec. 5.3 / 8.1) */
-    BANDLU_TC = 3       /* dgbtrf only, opt-in: window in FP64 tensor-core (DMMA) fragments, compiled
+    BANDLU_TC = 3,      /* dgbtrf only, opt-in: window in FP64 tensor-core (DMMA) fragments, compiled
                            (kl, ku) with kl+1 <= 16 (bandlu_tc_available); same LAPACK operation
                            sequence, bitwise equal results */
+    BANDLU_ROWS = 4     /* dgbtrf only: register window with R row slots per lane and block-preloaded
+                           band rows, compiled (kl, ku) only (bandlu_rows_available); AUTO prefers it
+                           where compiled; bitwise equal results */
 };
 
 /* ---- dgbtrf: band LU with partial pivoting ---- */
@@ -179,6 +182,8 @@ int bandlu_trs_variant(int n, int kl, int ku, int nrhs);
  * else 0 (no launch).  BANDLU_TC is never chosen by AUTO; force it with
  * dgbtrf_strided_batched_ex. */
 int bandlu_tc_available(int kl, int ku);
+/* 1 if a row-slot (BANDLU_ROWS) factorization kernel is compiled for (kl, ku), else 0. */
+int bandlu_rows_available(int kl, int ku);
 /* ABI version of this library. */
 int bandlu_version(void);
 

@@ -18,7 +18,7 @@ import torch
 
 from . import _build
 
-AUTO, GENERIC, WINDOW, TC = 0, 1, 2, 3
+AUTO, GENERIC, WINDOW, TC, ROWS = 0, 1, 2, 3, 4
 ERR_UNSUPPORTED, ERR_CUDA = 1000, 2000
 
 _lib = None
@@ -68,6 +68,7 @@ def load(build_if_missing: bool = False):
         "dgbtrfs_strided_batched_ex": [i, i, i, i, p, i, i64, p, i64, p, i, i64, p, i, p, i],
         "bandlu_trf_variant": [i, i, i, i],
         "bandlu_tc_available": [i, i],
+        "bandlu_rows_available": [i, i],
         "bandlu_trs_variant": [i, i, i, i],
         "bandlu_version": [],
     }
@@ -82,7 +83,7 @@ def load(build_if_missing: bool = False):
 # exported symbol list (checked by tests against include/bandlu.h)
 EXPORTS = ("dgbtrf_batched", "dgbtrf_strided_batched", "dgbtrf_strided_batched_ex", "dgbtrs_batched",
            "dgbtrs_strided_batched", "dgbtrs_strided_batched_ex", "dgbsv_batched", "dgbsv_strided_batched",
-           "dgbsv_strided_batched_host", "dgbtrfs_strided_batched", "dgbtrfs_strided_batched_ex", "bandlu_trf_variant", "bandlu_trs_variant", "bandlu_tc_available",
+           "dgbsv_strided_batched_host", "dgbtrfs_strided_batched", "dgbtrfs_strided_batched_ex", "bandlu_trf_variant", "bandlu_trs_variant", "bandlu_tc_available", "bandlu_rows_available",
            "bandlu_version")
 
 
@@ -206,6 +207,11 @@ def trf_variant(m: int, n: int, kl: int, ku: int) -> int:
 def tc_available(kl: int, ku: int) -> bool:
     """True if the opt-in tensor-core factorization (variant TC) is compiled for (kl, ku)."""
     return bool(load().bandlu_tc_available(kl, ku))
+
+
+def rows_available(kl: int, ku: int) -> bool:
+    """True if a row-slot factorization kernel (variant ROWS) is compiled for (kl, ku)."""
+    return bool(load().bandlu_rows_available(kl, ku))
 
 
 def trs_variant(n: int, kl: int, ku: int, nrhs: int) -> int:

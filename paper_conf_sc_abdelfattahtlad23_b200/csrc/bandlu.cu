@@ -11,6 +11,7 @@
 
 #include "../../include/bandlu.h"
 #include "common.cuh"
+#include "gbtrf_rows.cuh"
 #include "gbtrf_tc.cuh"
 #include "gbtrf_window.cuh"
 #include "gbtrs_window.cuh"
@@ -50,6 +51,29 @@ namespace {
 #endif
 #endif
 
+// (KL, KU, G, R): bands compiled as row-slot kernels (gbtrf_rows.cuh, G lanes x
+// R rows per matrix, block-preloaded incoming rows); a subset of the window
+// list (the solve launches reuse the window trs kernels).  AUTO prefers them.
+// Only bands where the kernel keeps the window kernel's matrices per warp
+// (G*R >= kl+1+4 with the same G) are listed; R = 2 (4 matrices per warp at
+// (10,10)) needs ~250 registers and measured slower.
+#ifndef BANDLU_ROWS_C3_G
+#define BANDLU_ROWS_C3_G 16
+#endif
+#ifndef BANDLU_ROWS_C3_R
+#define BANDLU_ROWS_C3_R 1
+#endif
+#if defined(BANDLU_NO_ROWS)
+#define BANDLU_ROWS_LIST(X)
+#elif defined(BANDLU_ONLY_C3)
+#define BANDLU_ROWS_LIST(X) X(10, 10, BANDLU_ROWS_C3_G, BANDLU_ROWS_C3_R)
+#else
+#define BANDLU_ROWS_LIST(X)                              \
+    X(10, 10, BANDLU_ROWS_C3_G, BANDLU_ROWS_C3_R)        \
+    X(10, 7, 16, 1)                                      \
+    X(2, 32, 8, 1)
+#endif
+
 // trs launch geometry: target resident warps (148 SMs x 8)
 constexpr int64_t kTrsWarpsTarget = 148 * 8;
 
@@ -77,6 +101,18 @@ int launch_trf_window(int m, int n, AP A, int ldab, PP P, int *info, int batch, 
     return cuda_ret(cudaGetLastError());
 }
 
+template <int KL, int KU, int G, int R, bool FWD, class AP, class PP, class BP>
+int launch_trf_rows(int m, int n, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st, BP B) {
+    using C = TrfRows<KL, KU, G, R>;
+    auto k = gbtrf_rows_kernel<KL, KU, G, R, FWD, AP, PP, BP>;
+    size_t sm = C::smem_bytes();
+    if (int r = set_smem(k, sm)) return r;
+    const int64_t per_block = (int64_t)C::WARPS * C::GPW;
+    const unsigned grid = (unsigned)((batch + per_block - 1) / per_block);
+    k<<<grid, C::WARPS * 32, sm, st>>>(m, n, A, ldab, P, info, batch, B);
+    return cuda_ret(cudaGetLastError());
+}
+
 template <class AP, class PP>
 int launch_trf_generic(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st) {
     const unsigned grid = (unsigned)(((int64_t)batch * 32 + 127) / 128);
@@ -88,6 +124,14 @@ bool trf_window_available(int kl, int ku) {
 #define X(a, b) \
     if (kl == a && ku == b) return true;
     BANDLU_WINDOW_LIST(X)
+#undef X
+    return false;
+}
+
+bool trf_rows_available(int kl, int ku) {
+#define X(a, b, g, r) \
+    if (kl == a && ku == b) return true;
+    BANDLU_ROWS_LIST(X)
 #undef X
     return false;
 }
@@ -104,6 +148,7 @@ int pick_trf(int m, int n, int kl, int ku) {
     if (m <= 0 || n <= 0) return BANDLU_GENERIC;
     // BANDLU_TC is opt-in: measured slower than the row-owner window at C3
     // (1.54 vs 1.10 ms), so AUTO never picks it.
+    if (trf_rows_available(kl, ku)) return BANDLU_ROWS;
     return trf_window_available(kl, ku) ? BANDLU_WINDOW : BANDLU_GENERIC;
 }
 
@@ -129,6 +174,13 @@ int run_trf(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int b
 #undef X
         return BANDLU_ERR_UNSUPPORTED;
     }
+    if (variant == BANDLU_ROWS && m > 0 && n > 0) {
+#define X(a, b, g, r) \
+    if (kl == a && ku == b) return launch_trf_rows<a, b, g, r, false>(m, n, A, ldab, P, info, batch, st, Strided<double>{nullptr, 0});
+        BANDLU_ROWS_LIST(X)
+#undef X
+        return BANDLU_ERR_UNSUPPORTED;
+    }
     if (variant == BANDLU_WINDOW && m > 0 && n > 0) {
 #define X(a, b) \
     if (kl == a && ku == b) return launch_trf_window<a, b, false>(m, n, A, ldab, P, info, batch, st, Strided<double>{nullptr, 0});
@@ -136,7 +188,8 @@ int run_trf(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int b
 #undef X
         return BANDLU_ERR_UNSUPPORTED;
     }
-    if (variant != BANDLU_GENERIC && variant != BANDLU_WINDOW && variant != BANDLU_TC) return BANDLU_ERR_UNSUPPORTED;
+    if (variant != BANDLU_GENERIC && variant != BANDLU_WINDOW && variant != BANDLU_TC && variant != BANDLU_ROWS)
+        return BANDLU_ERR_UNSUPPORTED;
     return launch_trf_generic(m, n, kl, ku, A, ldab, P, info, batch, st);
 }
 
@@ -220,6 +273,17 @@ int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ld
         int r = BANDLU_ERR_UNSUPPORTED;
         Strided<const double> Ac{A.base, A.stride};
         Strided<const int> Pc{P.base, P.stride};
+        if (trf_rows_available(kl, ku)) {
+#define X(a, b, g, rr)                                                                                    \
+    if (kl == a && ku == b) {                                                                             \
+        r = 0;                                                                                            \
+        if (phase != 2) r = launch_trf_rows<a, b, g, rr, true>(n, n, A, ldab, P, info, batch, st, B);     \
+        if (r == 0 && phase != 1) r = launch_trs_window<a, b>(n, 1, Ac, ldab, Pc, B, ldb, nullptr, batch, st, 0); \
+    }
+            BANDLU_ROWS_LIST(X)
+#undef X
+            return r;
+        }
 #define X(a, b)                                                                                           \
     if (kl == a && ku == b) {                                                                             \
         r = 0;                                                                                            \
@@ -305,6 +369,7 @@ int bandlu_version(void) { return 1; }
 
 int bandlu_trf_variant(int m, int n, int kl, int ku) { return pick_trf(m, n, kl, ku); }
 int bandlu_tc_available(int kl, int ku) { return trf_tc_available(kl, ku) ? 1 : 0; }
+int bandlu_rows_available(int kl, int ku) { return trf_rows_available(kl, ku) ? 1 : 0; }
 int bandlu_trs_variant(int n, int kl, int ku, int nrhs) { return pick_trs(n, kl, ku, nrhs); }
 
 int dgbtrf_strided_batched_ex(int m, int n, int kl, int ku, double *dA, int ldab, int64_t strideA, int *dipiv,

@@ -113,6 +113,14 @@ __device__ __forceinline__ double ld_shared_f64(uint32_t a) {
     return v;
 }
 
+// volatile: ptxas may not merge neighbouring loads into one 128-bit access
+// (a 64-bit broadcast read costs one wavefront for all groups of a warp)
+__device__ __forceinline__ double ld_volatile_shared_f64(uint32_t a) {
+    double v;
+    asm volatile("ld.volatile.shared.f64 %0, [%1];\n" : "=d"(v) : "r"(a) : "memory");
+    return v;
+}
+
 // ---- mbarrier + bulk (TMA 1D) copies
 __device__ __forceinline__ void mbar_init(uint32_t bar, unsigned count) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(bar), "r"(count) : "memory");

@@ -1,0 +1,358 @@
+// gbtrf_rows.cuh -- sm_100a band LU with partial pivoting, R row slots per
+// lane, the incoming rows of a block preloaded into free slots.
+//
+// What it computes: LAPACK DGBTF2 exactly (Sec. 5.1 pseudo-code
+// P:350-367, ju rule P:492-494, right-only swaps P:358/P:369-374), the same
+// fp64 operation sequence as the oracle => bitwise-equal factors, ipiv, info.
+//
+// Why a second register-window kernel: the row-owner
+// window (gbtrf_window.cuh) is bounded by the shared-memory pipe -- per
+// matrix-column step ~42 wavefronts: the pivot row written to a record by one
+// lane, read back by the 16 lanes of the matrix with 128-bit loads, and the
+// next band row loaded by the retiring pivot lane alone.  Measured on B200
+// (tools/probes/lsu_probe4.cu): a broadcast LDS.64 costs one cycle per warp
+// whatever the number of distinct addresses (<= 128 B), a 1-lane LDS.128 two.
+// So this kernel
+//  * packs more matrices into a warp: G lanes per matrix hold R rows each
+//    (G*R >= KL+1+U slots; C3 (10,10): G = 8, R = 2 -> 4 matrices per warp,
+//    one broadcast read serves all four);
+//  * broadcasts the pivot row with 64-bit loads (one per column);
+//  * loads a block's U incoming band rows at block start, all at once, into
+//    the slots freed by the previous block's pivot rows (ballot + rank), so
+//    no lane reloads its registers inside the column step.  A preloaded row
+//    is not a pivot candidate until its step (pos <= j + KL); before that its
+//    multiplier is forced to 0 (its column-j entry is a structural zero), so
+//    it receives no update -- exactly DGBTF2, where that row is outside the
+//    active window.
+// Interchanges are relabelings (reading 10), IAMAX is first-max
+// (exact 64-bit key compare, ties by smallest logical row; reading 2).
+#pragma once
+#include "common.cuh"
+
+#ifndef BANDLU_ROWS_WARPS
+#define BANDLU_ROWS_WARPS 4
+#endif
+
+namespace bandlu {
+
+template <int KL_, int KU_, int G_, int R_>
+struct TrfRows {
+    static constexpr int KL = KL_, KU = KU_, KV = KL + KU, W = KV + 1;
+    static constexpr int G = G_, R = R_, GPW = 32 / G;
+    static constexpr int U = 4;                  // columns per block (window shift granularity)
+    static constexpr int WS = W + U, H = (WS + 1) / 2;
+    static_assert(G * R >= KL + 1 + U, "slots: KL+1 active rows + U preloaded rows");
+    static_assert(32 % G == 0, "group size");
+    // ring row / record pitch (doubles), spare pair at RP: (B entry[, logical row])
+    static constexpr int WP = (G >= 8) ? ((2 * H + 2 + 11) / 16) * 16 + 4 : 2 * H + 2 + ((2 * H + 2) % 4 == 2 ? 0 : 2);
+    static constexpr int RP = WP - 2;
+    static constexpr int D = 4, DB = D / U;      // staging lead (rows / blocks)
+    static constexpr int RR = pow2_ceil((DB + 1) * U);
+    static constexpr int NREC = U;
+    // group pitch == 2 (mod 16) doubles: the GPW groups of a warp read their
+    // records at the same offsets, so their 64-bit broadcasts must sit in
+    // distinct banks (a multiple of 128 B would make them a GPW-way conflict)
+    static constexpr int GROUP_DBL = ((RR + NREC) * WP + 13) / 16 * 16 + 2;
+    static constexpr int BK = W + U - 1;
+    static constexpr int BIT = (BK * U + G - 1) / G;
+    static_assert(BIT <= 32, "block element mask");
+    static constexpr int WARPS_FIT = (72 * 1024) / (GPW * GROUP_DBL * 8);
+    static constexpr int WARPS = WARPS_FIT < 1 ? 1 : (WARPS_FIT < BANDLU_ROWS_WARPS ? WARPS_FIT : BANDLU_ROWS_WARPS);
+#ifndef BANDLU_ROWS_MINW
+#define BANDLU_ROWS_MINW 12
+#endif
+    // resident warps per SM target (wide windows: 8, as the window kernel)
+    static constexpr int MINB = ((W <= 24 ? BANDLU_ROWS_MINW : 8) + WARPS - 1) / WARPS;
+    static constexpr size_t smem_bytes() { return (size_t)WARPS * GPW * GROUP_DBL * sizeof(double); }
+};
+
+// max of a 32-bit value over the G lanes of each group (all 32 lanes call)
+template <int G>
+__device__ __forceinline__ unsigned group_max_u32(unsigned v, int g) {
+    if constexpr (G == 32) {
+        return __reduce_max_sync(0xffffffffu, v);
+    } else if constexpr (G == 16) {
+        const unsigned m0 = __reduce_max_sync(0xffffffffu, g == 0 ? v : 0u);
+        const unsigned m1 = __reduce_max_sync(0xffffffffu, g == 1 ? v : 0u);
+        return g == 0 ? m0 : m1;
+    } else {
+#pragma unroll
+        for (int off = 1; off < G; off <<= 1) v = max(v, __shfl_xor_sync(0xffffffffu, v, off));
+        return v;
+    }
+}
+template <int G>
+__device__ __forceinline__ unsigned group_min_u32(unsigned v) {
+#pragma unroll
+    for (int off = 1; off < G; off <<= 1) v = min(v, __shfl_xor_sync(0xffffffffu, v, off));
+    return v;
+}
+
+template <int KL, int KU, int G, int R, bool FWD, class AP, class PP, class BP>
+__global__ void __launch_bounds__(TrfRows<KL, KU, G, R>::WARPS * 32, TrfRows<KL, KU, G, R>::MINB)
+    gbtrf_rows_kernel(int m, int n, AP A, int ldab, PP P, int *__restrict__ info, int batch, BP Bv) {
+    using C = TrfRows<KL, KU, G, R>;
+    constexpr int KV = C::KV, U = C::U, H = C::H, WP = C::WP, RP = C::RP, D = C::D, RR = C::RR, BK = C::BK,
+                  BIT = C::BIT;
+    constexpr int FREE = 0x7fffffff;
+    extern __shared__ __align__(16) double smem[];
+
+    const int lane = (int)lane_id(), wib = (int)(threadIdx.x >> 5);
+    const int g = lane / G, t = lane % G;
+    const int64_t mat = ((int64_t)blockIdx.x * C::WARPS + wib) * C::GPW + g;
+    const bool live = mat < batch;
+    if (__ballot_sync(0xffffffffu, live) == 0u) return;
+
+    double *__restrict__ ab = live ? A.get(mat) : nullptr;
+    int *__restrict__ ipiv = live ? P.get(mat) : nullptr;
+    double *__restrict__ bv = (FWD && live) ? Bv.get(mat) : nullptr;
+    if (m <= 0 || n <= 0) {
+        if (live && t == 0) info[mat] = 0;
+        return;
+    }
+    const int mloc = live ? m : 0;
+    double *ring = smem + (size_t)(wib * C::GPW + g) * C::GROUP_DBL;
+    const uint32_t ring_s = smem_u32(ring);
+    const uint32_t rec_s = ring_s + RR * WP * 8;
+    const double *safe = live ? ab : g_dummy;
+
+    // Ring row of input row q holds A(q, q-KL+c) at position o+1+c
+    // (o = (q-KL-1) % U, fixed per ring row), zeros elsewhere.
+    for (int i = t; i < RR * WP; i += G) ring[i] = 0.0;
+    __syncwarp();
+
+    // ---- block transfers: element e = t + k*G -> row offset bs = e % U, column offset bk = e / U
+    const int bo0 = (t / U) * (ldab - 1) + (t % U), bstep = (G / U) * (ldab - 1);
+    auto boff = [&](int k) -> int {
+        if constexpr (G % U == 0) return bo0 + k * bstep;
+        const int e = t + k * G;
+        return (e / U) * (ldab - 1) + (e % U);
+    };
+    unsigned bmask = 0;
+#pragma unroll
+    for (int k = 0; k < BIT; ++k) {
+        const int e = t + k * G, bs = e % U, bk = e / U;
+        if (bk < BK && bk - bs >= 0 && bk - bs <= KV) bmask |= 1u << k;
+    }
+    auto stage_block = [&](int qb, const double *colq) {
+#pragma unroll
+        for (int k = 0; k < BIT; ++k) {
+            const int e = t + k * G, bs = e % U, bk = e / U;
+            if (bmask >> k & 1u) {
+                const int q = qb + bs;
+                const bool ok = (q < mloc) && (qb - KL + bk < n);
+                const uint32_t dst = ring_s + (uint32_t)(((q & (RR - 1)) * WP + 1 + bk) * 8);
+                cp_async8(dst, ok ? colq + boff(k) + (KV + KL) : safe, ok ? 8u : 0u);
+            }
+        }
+        if constexpr (FWD) {
+#pragma unroll
+            for (int i = t; i < U; i += G) {
+                const int q = qb + i;
+                const bool okb = (q < mloc);
+                const uint32_t dstb = ring_s + (uint32_t)(((q & (RR - 1)) * WP + RP) * 8);
+                cp_async8(dstb, okb ? (const void *)(bv + q) : (const void *)safe, okb ? 8u : 0u);
+            }
+        }
+        cp_async_commit();
+    };
+#pragma unroll 1
+    for (int d = 0; d < C::DB; ++d) stage_block(KL + 1 + d * U, live ? ab + (int64_t)(1 + d * U) * ldab : g_dummy);
+    const double *scol = live ? ab + (int64_t)(1 + D) * ldab : g_dummy;
+
+    // ---- window registers: slot r of row slot i = column j0 + r; rows 0..KL in slots i = ri*G + t
+    double2 v[R][H];
+    int pos[R];
+    double bq[R];
+#define VS(ri, k) (((k) & 1) ? v[ri][(k) >> 1].y : v[ri][(k) >> 1].x)
+#pragma unroll
+    for (int ri = 0; ri < R; ++ri) {
+        const int i = ri * G + t;
+        const bool row_ok = live && (i <= KL) && (i < m);
+#pragma unroll
+        for (int h = 0; h < H; ++h) {
+            const int c0 = 2 * h, c1 = 2 * h + 1;
+            const bool ok0 = row_ok && (c0 < n) && (c0 <= i + KU);
+            const bool ok1 = row_ok && (c1 < n) && (c1 <= i + KU);
+            v[ri][h].x = ok0 ? ab[(int64_t)c0 * ldab + (KV + i - c0)] : 0.0;
+            v[ri][h].y = ok1 ? ab[(int64_t)c1 * ldab + (KV + i - c1)] : 0.0;
+        }
+        pos[ri] = (live && i <= KL) ? i : FREE;
+        bq[ri] = 0.0;
+        if constexpr (FWD) bq[ri] = row_ok ? bv[i] : 0.0;
+    }
+
+    int linfo = 0;
+    const int mn = min(m, n);
+    double *colj = live ? ab + KV : nullptr;  // &AB(KV, j)
+    double *colb = live ? ab : nullptr;       // &AB(0, j0)
+    int *ipj = ipiv;
+    const unsigned gbits = (G == 32) ? 0xffffffffu : ((1u << G) - 1u);
+    const unsigned gbase = (unsigned)(g * G);
+    const unsigned below = (1u << t) - 1u;
+#pragma unroll 1
+    for (int j0 = 0; j0 < mn; j0 += U) {
+        cp_async_wait<C::DB - 1>();  // rows j0+KL+1 .. j0+KL+U landed (this lane's part)
+        __syncwarp();
+        // ---- preload rows j0+KL+1+o (o = 0..U-1) into the first U free slots of the group
+        {
+            int before = 0;
+#pragma unroll
+            for (int ri = 0; ri < R; ++ri) {
+                const bool fr = (pos[ri] == FREE) || (pos[ri] >= mloc);
+                const unsigned fb = (__ballot_sync(0xffffffffu, fr) >> gbase) & gbits;
+                const int rank = before + __popc(fb & below);
+                const bool take = fr && rank < U;
+                const int q = j0 + KL + 1 + rank;
+                const uint32_t rr = ring_s + (uint32_t)((q & (RR - 1)) * WP * 8);
+#pragma unroll
+                for (int h = 0; h < H; ++h) ld_shared_v2_if(take, rr + h * 16, v[ri][h]);
+                if constexpr (FWD) ld_shared_f64_if(take, rr + RP * 8, bq[ri]);
+                if (take) pos[ri] = q;
+                before += __popc(fb);
+            }
+        }
+        stage_block(j0 + KL + 1 + D, scol);
+        scol += (int64_t)U * ldab;
+#pragma unroll
+        for (int s = 0; s < U; ++s) {  // column j = j0 + s sits in slot s
+            const int j = j0 + s;
+            if (j >= mn) break;
+
+            // ---- IAMAX over the candidates (logical rows j..min(j+KL, m-1))
+            double x[R];
+            bool cand[R];
+            uint64_t kb = 0;
+            int pb = FREE, rb = 0;
+            bool cb = false;
+#pragma unroll
+            for (int ri = 0; ri < R; ++ri) {
+                x[ri] = VS(ri, s);
+                cand[ri] = (pos[ri] <= j + KL) && (pos[ri] < mloc);
+                const uint64_t k = cand[ri] ? abs_key(x[ri]) : 0ull;
+                const bool better = cand[ri] && (!cb || k > kb || (k == kb && pos[ri] < pb));
+                if (better) {
+                    kb = k;
+                    pb = pos[ri];
+                    rb = ri;
+                    cb = true;
+                }
+            }
+            const unsigned hi = (unsigned)(kb >> 32);
+            const unsigned mhi = group_max_u32<G>(hi, g);
+            unsigned gb = (__ballot_sync(0xffffffffu, cb && hi == mhi) >> gbase) & gbits;
+            if (__any_sync(0xffffffffu, live && __popc(gb) != 1)) {
+                // exact tie-break: low word, then smallest logical row (first index)
+                const unsigned lo = (unsigned)kb;
+                const unsigned mlo = group_max_u32<G>((cb && hi == mhi) ? lo : 0u, g);
+                const unsigned pp = group_min_u32<G>((cb && hi == mhi && lo == mlo) ? (unsigned)pb : 0xffffffffu);
+                gb = (__ballot_sync(0xffffffffu, cb && (unsigned)pb == pp) >> gbase) & gbits;
+            }
+            const bool is_piv = (t == __ffs(gb) - 1);
+
+            // ---- pivot row (U row j: slots s..s+KV) + (B entry, logical row) -> record s
+            const uint32_t rcs = rec_s + (uint32_t)(s * WP * 8);
+#pragma unroll
+            for (int ri = 0; ri < R; ++ri) {
+#pragma unroll
+                for (int h = s / 2; h <= (s + KV) / 2; ++h) st_shared_v2_if(is_piv && rb == ri, rcs + h * 16, v[ri][h]);
+            }
+            {
+                double bsel = bq[0];
+#pragma unroll
+                for (int ri = 1; ri < R; ++ri) bsel = (rb == ri) ? bq[ri] : bsel;
+                st_shared_v2_if(is_piv, rcs + RP * 8, make_double2(bsel, __longlong_as_double((long long)pb)));
+            }
+            __syncwarp();
+
+            // ---- broadcast read (64-bit: one cycle per warp for all groups)
+            const double2 yp = ld_shared_v2(rcs + RP * 8);
+            const int ppos = (int)__double_as_longlong(yp.y);
+            const double p = ld_volatile_shared_f64(rcs + s * 8);
+            const bool zp = (p == 0.0);
+            if (is_piv) *ipj = ppos + 1;
+            if (live && zp && linfo == 0) linfo = j + 1;
+
+            // ---- interchange = relabel; the pivot slot retires after this step
+            bool pslot[R];
+#pragma unroll
+            for (int ri = 0; ri < R; ++ri) {
+                pslot[ri] = is_piv && rb == ri;
+                if (live && pos[ri] == j && !pslot[ri]) pos[ri] = ppos;  // dead groups: no record was written
+            }
+
+            // ---- SCAL: multiplier = x * RN(1/p) (DSCAL(ONE/pivot), Q7)
+            const double rinv = __drcp_rn(p);
+            double lu[R];
+#pragma unroll
+            for (int ri = 0; ri < R; ++ri) {
+                const double l = zp ? x[ri] : __dmul_rn(x[ri], rinv);
+                lu[ri] = (cand[ri] && !zp) ? l : 0.0;
+                if (cand[ri] && !pslot[ri]) colj[pos[ri] - j] = l;
+            }
+            if constexpr (FWD) {
+                const double y = yp.x;
+                if (is_piv) bv[j] = y;
+                if (y != 0.0) {
+#pragma unroll
+                    for (int ri = 0; ri < R; ++ri) bq[ri] = __fma_rn(lu[ri], -y, bq[ri]);
+                }
+            }
+            // ---- RANK-1 update of the window columns j+1..j+KV (DGER, alpha = -1, FMA)
+#pragma unroll
+            for (int k = 1; k <= KV; ++k) {
+                const double uk = ld_volatile_shared_f64(rcs + (s + k) * 8);
+#pragma unroll
+                for (int ri = 0; ri < R; ++ri) VS(ri, s + k) = __fma_rn(lu[ri], -uk, VS(ri, s + k));
+            }
+#pragma unroll
+            for (int ri = 0; ri < R; ++ri)
+                if (pslot[ri]) pos[ri] = FREE;
+            colj += ldab;
+            ++ipj;
+        }
+        // ---- U rows j0 .. j0+U-1 (the block's records) -> HBM, 32-byte column chunks
+        __syncwarp();
+#pragma unroll
+        for (int k = 0; k < BIT; ++k) {
+            const int e = t + k * G, bs = e % U, bk = e / U;
+            if (live && (bmask >> k & 1u) && j0 + bs < mn && j0 + bk < n)
+                colb[boff(k) + KV] = ld_shared_f64(rec_s + (uint32_t)((bs * WP + bk) * 8));
+        }
+        colb += (int64_t)U * ldab;
+        __syncwarp();
+        // shift the window by U columns: slot r <- slot r+U
+#pragma unroll
+        for (int ri = 0; ri < R; ++ri) {
+#pragma unroll
+            for (int h = 0; h < H; ++h) {
+                if (h + U / 2 < H) {
+                    v[ri][h] = v[ri][h + U / 2];
+                } else {
+                    v[ri][h].x = 0.0;
+                    v[ri][h].y = 0.0;
+                }
+            }
+        }
+    }
+    cp_async_wait<0>();
+    __syncwarp();
+#undef VS
+    if (!live) return;
+
+    // LAPACK's SET_FILLIN also zeroes fill-row positions whose matrix row is
+    // >= m when m < n (those rows are never pivot rows here).
+    if (m < n) {
+        for (int c = m + KU + 1 + t; c <= min(n - 1, m + KV - 1); c += G) {
+#pragma unroll 1
+            for (int r = 0; r < KL; ++r) {
+                const int i = c - KV + r;
+                const bool zeroed = (c >= KU + 1 && c <= min(KV, n) - 1 && r >= KV - c) || (c >= KV && c - KV < mn);
+                if (i >= m && zeroed) ab[(int64_t)c * ldab + r] = 0.0;
+            }
+        }
+    }
+    if (t == 0) info[mat] = linfo;
+}
+
+}  // namespace bandlu

@@ -108,7 +108,8 @@ def test_gbsv_argument_errors(lib):
 
 def test_variant_heuristic_is_shape_only(lib):
     from paper_conf_sc_abdelfattahtlad23_b200 import binding as b
-    assert b.trf_variant(512, 512, 10, 10) == b.WINDOW
+    assert b.trf_variant(512, 512, 10, 10) == b.ROWS
+    assert b.rows_available(10, 10) and b.rows_available(2, 32) and not b.rows_available(1, 1)
     assert b.tc_available(10, 10) and not b.tc_available(1, 1)  # opt-in tensor-core kernel
     assert b.trf_variant(256, 256, 1, 1) == b.WINDOW
     assert b.trf_variant(100, 100, 32, 32) == b.GENERIC  # kl+1 > 32 lanes: safeguard kernel

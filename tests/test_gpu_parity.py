@@ -36,8 +36,11 @@ def _gpu_trf(A_np, m, n, kl, ku, variant=bl.AUTO):
 
 def trf_variants(kl, ku):
     """Forced factorization variants to cross-check: the safeguard, the row-owner
-    window, and the tensor-core (DMMA) kernel where it is compiled for (kl, ku)."""
+    window, and the row-slot (ROWS) and tensor-core (DMMA) kernels where they are
+    compiled for (kl, ku)."""
     v = [bl.WINDOW, bl.GENERIC]
+    if bl.rows_available(kl, ku):
+        v.append(bl.ROWS)
     if bl.tc_available(kl, ku):
         v.append(bl.TC)
     return v
@@ -56,7 +59,7 @@ def _check_trf(m, n, kl, ku, batch, variant, ldab=None, first=0, A_in=None):
 
 
 @pytest.mark.parametrize("kl,ku", WINDOW_BANDS)
-@pytest.mark.parametrize("variant", [bl.WINDOW, bl.GENERIC, bl.TC])
+@pytest.mark.parametrize("variant", [bl.WINDOW, bl.GENERIC, bl.ROWS, bl.TC])
 @pytest.mark.parametrize("n", [1, 2, 7, 37, 100])
 def test_trf_parity_small(kl, ku, variant, n):
     if variant not in trf_variants(kl, ku):
@@ -76,7 +79,7 @@ def test_trf_parity_rectangular(kl, ku, mn):
 @pytest.mark.parametrize("kl,ku", [(2, 3), (10, 10), (5, 9), (33, 20), (32, 32), (40, 64), (0, 40)])
 def test_trf_parity_generic_any_band(kl, ku):
     _check_trf(150, 150, kl, ku, batch=11, variant=bl.GENERIC)
-    assert bl.trf_variant(150, 150, kl, ku) in (bl.GENERIC, bl.WINDOW)
+    assert bl.trf_variant(150, 150, kl, ku) in (bl.GENERIC, bl.WINDOW, bl.ROWS)
 
 
 @pytest.mark.parametrize("kl,ku", [(1, 1), (10, 10), (2, 32)])
@@ -346,3 +349,14 @@ def test_application_shaped_workloads(batch, n, kl, ku):
     assert np.array_equal(P.cpu().numpy(), ipo)
     assert np.all(same_bits(Ag.cpu().numpy(), Ao))
     assert np.all(same_bits(Bg.cpu().numpy(), Bo))
+
+
+@pytest.mark.parametrize("kl,ku", [(10, 10), (2, 32), (10, 7)])
+def test_trf_batch_tail_after_other_launches(kl, ku):
+    """Batch tails leave dead matrix groups in the last CTA; they must not act on
+    shared memory left over by earlier launches (regression: a dead group once
+    relabelled a row from a never-written pivot record)."""
+    for variant in trf_variants(kl, ku):
+        _check_trf(300, 300, kl, ku, batch=97, variant=variant)  # fills shared memory with live data
+        for batch in (1, 3, 5):
+            _check_trf(90, 90, kl, ku, batch=batch, variant=variant, first=batch)

@@ -18,6 +18,6 @@ print('trf factors ok', ok.all(), 'bad', (~ok).sum(), 'ipiv ok', np.array_equal(
 if m == n:
     B = I.gen_rhs(n, nrhs, count=batch); Bo = B.copy(); oracle.dgbtrs(Ao, ipo, Bo, n, kl, ku)
     Bg = torch.from_numpy(B).cuda()
-    bl.dgbtrs_strided_batched('N', n, kl, ku, torch.from_numpy(Ao).cuda(), torch.from_numpy(ipo).cuda(), Bg, variant=variant)
+    bl.dgbtrs_strided_batched('N', n, kl, ku, torch.from_numpy(Ao).cuda(), torch.from_numpy(ipo).cuda(), Bg, variant=variant if variant in (1, 2) else 0)
     torch.cuda.synchronize()
     print('trs ok', same(Bg.cpu().numpy(), Bo).all())
