@@ -200,13 +200,14 @@ int launch_trs_window(int n, int nrhs, AP A, int ldab, PP P, BP B, int ldb, cons
     using C = TrsWin<KL, KU>;
     const int R = nrhs >= 32 ? 32 : pow2_ceil(nrhs);
     const int chunks = (nrhs + 31) / 32;
-    auto k = gbtrs_window_kernel<KL, KU, AP, PP, BP>;
+    const bool pairs = R >= 2;
+    auto k = pairs ? gbtrs_window_kernel<KL, KU, true, AP, PP, BP> : gbtrs_window_kernel<KL, KU, false, AP, PP, BP>;
     const int64_t units = (int64_t)batch * chunks;
     // Each lane runs a long serial chain: spread the units over >= ~8 warps per
     // SM (all four schedulers busy) before packing more of them into a warp.
     int gpw = 32 / R;
     while (gpw > 1 && units < (int64_t)gpw * kTrsWarpsTarget) gpw >>= 1;
-    const size_t sm = C::smem_bytes(R, gpw);
+    const size_t sm = C::smem_bytes(R, gpw, pairs);
     if (int r = set_smem(k, sm)) return r;
     const unsigned grid = (unsigned)((units + gpw - 1) / gpw);
     k<<<grid, 32, sm, st>>>(n, nrhs, A, ldab, P, B, ldb, skip, batch, R, chunks, gpw, fwd);
