@@ -75,7 +75,10 @@ namespace {
 #endif
 
 // trs launch geometry: target resident warps (148 SMs x 8)
-constexpr int64_t kTrsWarpsTarget = 148 * 8;
+#ifndef BANDLU_TRS_WPSM
+#define BANDLU_TRS_WPSM 8
+#endif
+constexpr int64_t kTrsWarpsTarget = 148 * BANDLU_TRS_WPSM;
 
 inline int cuda_ret(cudaError_t e) { return e == cudaSuccess ? 0 : BANDLU_ERR_CUDA + (int)e; }
 

@@ -42,6 +42,12 @@
 #include "common.cuh"
 
 // Tuning knobs (compile-time; overridable with -D for experiments)
+#ifndef BANDLU_TRF_D_NARROW
+#define BANDLU_TRF_D_NARROW 8
+#endif
+#ifndef BANDLU_TRF_G_NARROW
+#define BANDLU_TRF_G_NARROW 8
+#endif
 #ifndef BANDLU_TRF_U
 #define BANDLU_TRF_U 4
 #endif
@@ -78,9 +84,13 @@ struct TrfWin {
     static constexpr int RP = WP - 2;
     // lanes per matrix: pow2 >= KL+1; wide windows use >= 8 so that a warp's
     // smem rings (and so the resident warps per SM) stay within budget
-    static constexpr int G = pow2_ceil(KL + 1) < (W > 24 ? 8 : 1) ? (W > 24 ? 8 : 1) : pow2_ceil(KL + 1);
+    // (narrow bands: >= BANDLU_TRF_G_NARROW lanes, so that a batch spreads over more warps)
+    static constexpr int GMIN = W > 24 ? 8 : (W <= 5 ? BANDLU_TRF_G_NARROW : 1);
+    static constexpr int G = pow2_ceil(KL + 1) < GMIN ? GMIN : pow2_ceil(KL + 1);
     static constexpr int GPW = 32 / G;           // matrices per warp
-    static constexpr int D = BANDLU_TRF_D;       // staging lead (rows, multiple of U)
+    // staging lead (rows, multiple of U): narrow bands do little work per step, so the
+    // HBM latency of a block's rows must be covered by more steps ahead
+    static constexpr int D = (W <= 5) ? BANDLU_TRF_D_NARROW : BANDLU_TRF_D;
     static constexpr int DB = D / U;             // staging lead in blocks
     static constexpr int RR = pow2_ceil((DB + 1) * U);  // ring rows (power of 2, multiple of U)
     static constexpr int NREC = U;               // pivot-row records: this block's U rows

@@ -36,19 +36,24 @@
 #pragma once
 #include "common.cuh"
 
+#ifndef BANDLU_TRS_NS_NARROW
+#define BANDLU_TRS_NS_NARROW 16
+#endif
+
 namespace bandlu {
 
 template <int KL_, int KU_>
 struct TrsWin {
     static constexpr int KL = KL_, KU = KU_, KV = KL + KU;
     static constexpr int WF = KL + 1, WB = KV + 1;         // forward / backward window lengths
-    static constexpr int NS = 8;                           // ring depth (column steps in flight)
+    // ring depth (column steps in flight): narrow bands need more steps to cover HBM latency
+    static constexpr int NS = (WB <= 5) ? BANDLU_TRS_NS_NARROW : 8;
     static constexpr int FMAX = (KL > WB ? KL : WB) + 2;   // factor doubles per slot (+16 B rounding)
     static constexpr int SP = (FMAX + 1) & ~1;             // even -> 16 B aligned slots
     // slot: [SP factor doubles][ipiv int, pad][R rhs doubles when rows move one per step]
     __host__ __device__ static constexpr int slot_dbl(int R, bool pairs) { return SP + 2 + (pairs ? 0 : (R + 1) & ~1); }
     static constexpr int AHEAD = (NS + 2) / 2;             // RHS pairs in flight (2*AHEAD-1 >= NS steps)
-    static constexpr int RPN = 8;                          // RHS pair ring depth (>= AHEAD + 1, power of 2)
+    static constexpr int RPN = pow2_ceil(AHEAD + 1);       // RHS pair ring depth (power of 2)
     // group: [NS slots][RPN pairs x R lanes x 2 doubles]; pitch == 2 (mod 4) doubles so that the
     // groups' broadcast reads of the same slot offset sit in different banks
     __host__ __device__ static constexpr int group_dbl(int R, bool pairs) {
