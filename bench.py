@@ -44,7 +44,11 @@ CONFIGS = {  # name: (batch per GPU, n, kl, ku, nrhs, description)
     # application-shaped batches (bands synthetic; the paper gives sizes only)
     "XGC": (512, 193, 4, 4, 1, "f4 XGC-like: batch=512, n=193 (P:226-227), kl=ku=4, nrhs=1"),
     "PELE": (10000, 50, 10, 10, 1, "f4 PELE-like: batch=10000, n=50 (P:195-197, 'many <= 50'), kl=ku=10, nrhs=1"),
+    # configs[4]: the n sweep, batch per point sized from free HBM (run_sweep)
+    "C5": (0, 0, 0, 0, 1, "configs[4]: n sweep 32-2048, (kl,ku) in {(2,3),(10,7),(32,32)}, batch filling HBM"),
 }
+C5_BANDS = ((2, 3), (10, 7), (32, 32))
+C5_NS = (32, 64, 128, 256, 512, 1024, 2048)
 
 
 def peaks():
@@ -137,6 +141,103 @@ def cpu_oracle_rate(n, kl, ku, nrhs, seconds=6.0, sample=None):
     return sample / best, sample, threads, reps
 
 
+def run_sweep(args, rank, world):
+    """configs[4]: n = 32..2048 x (kl, ku) in C5_BANDS; per point the
+    per-GPU batch fills --fill of free HBM (pristine copy + working copy of A and B),
+    weak scaling over ranks.  A seeded block of <= 256 MB is generated per point and
+    replicated on the device to the batch (identical per-matrix work; counter-based
+    inputs keep every replica bitwise reproducible).  One JSON line: value = total
+    nominal flops / total time over the sweep, per-point results under "sweep"."""
+    import torch
+    import torch.distributed as dist
+    import paper_conf_sc_abdelfattahtlad23_b200 as bl
+    from paper_conf_sc_abdelfattahtlad23_b200 import dist as bd
+    from paper_conf_sc_abdelfattahtlad23_b200 import inputs as I
+
+    rank, world, dev = bd.init("nccl")
+    bl.load()
+    st = torch.cuda.current_stream()
+    free = torch.cuda.mem_get_info(dev)[0]
+    points, tot_flop, tot_ms, tot_bytes = [], 0.0, 0.0, 0.0
+    sampler = ClockSampler(torch.cuda.current_device()) if rank == 0 else None
+    if sampler:
+        sampler.start()
+    for kl, ku in C5_BANDS:
+        for n in C5_NS:
+            ldab = 2 * kl + ku + 1
+            per = 2 * 8 * ldab * n + 2 * 8 * n + 4 * n + 4
+            bpg = max(1, int(args.fill * free / per))
+            gen = max(1, min(bpg, (256 << 20) // (8 * ldab * n)))
+            lo, _ = I.shard_range(bpg * world, rank, world)
+            blk_a = torch.from_numpy(I.gen_band(n, n, kl, ku, count=gen, first=lo)).to(dev)
+            blk_b = torch.from_numpy(I.gen_rhs(n, 1, count=gen, first=lo)).to(dev)
+            reps = (bpg + gen - 1) // gen
+            A0 = blk_a.repeat(reps, 1, 1)[:bpg].contiguous()
+            B0 = blk_b.repeat(reps, 1, 1)[:bpg].contiguous()
+            del blk_a, blk_b
+            A, B = torch.empty_like(A0), torch.empty_like(B0)
+            P = torch.zeros((bpg, n), dtype=torch.int32, device=dev)
+            info = torch.zeros(bpg, dtype=torch.int32, device=dev)
+
+            def step(evs=None):
+                A.copy_(A0)
+                B.copy_(B0)
+                if evs is not None:
+                    evs[0].record(st)
+                bl.dgbtrfs_strided_batched(n, kl, ku, A, P, B, info, phase=1)
+                if evs is not None:
+                    evs[1].record(st)
+                bl.dgbtrfs_strided_batched(n, kl, ku, A, P, B, info, phase=2)
+                if evs is not None:
+                    evs[2].record(st)
+
+            for _ in range(args.warmup):
+                step()
+            torch.cuda.synchronize()
+            assert int(info.abs().sum()) == 0
+            evs = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.steps)]
+            if world > 1:
+                dist.barrier()
+            torch.cuda.synchronize()
+            for k in range(args.steps):
+                step(evs[k])
+            torch.cuda.synchronize()
+            trf = sum(e[0].elapsed_time(e[1]) for e in evs) / args.steps
+            trs = sum(e[1].elapsed_time(e[2]) for e in evs) / args.steps
+            ms, trf, trs = bd.max_over_ranks([trf + trs, trf, trs], dev)
+            f_trf, f_trs = I.nominal_flops(n, kl, ku, 1)
+            b_trf, b_trs = I.alg_bytes(n, n, kl, ku, 1)
+            glob = bpg * world
+            points.append({"n": n, "kl": kl, "ku": ku, "batch_per_gpu": bpg, "ms_per_step": ms, "trf_ms": trf,
+                           "trs_ms": trs, "gflops": glob * (f_trf + f_trs) / (ms * 1e-3) / 1e9,
+                           "hbm_gbs": glob * (b_trf + b_trs) / (ms * 1e-3) / 1e9,
+                           "matrices_per_s": glob / (ms * 1e-3), "variant_trf": bl.trf_variant(n, n, kl, ku)})
+            tot_flop += glob * (f_trf + f_trs)
+            tot_bytes += glob * (b_trf + b_trs)
+            tot_ms += ms
+            del A0, B0, A, B, P, info
+            torch.cuda.empty_cache()
+    clocks = sampler.stop() if sampler else None
+    if rank == 0:
+        peak, peak_kind = peaks()
+        best = max(points, key=lambda q: q["hbm_gbs"])
+        line = {"metric": METRIC, "value": tot_flop / (tot_ms * 1e-3) / 1e9, "unit": "GFLOP/s", "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot_ms, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+                "data": "synthetic (seeded counter-based U(-1,1) bands, <=256 MB block replicated per point)",
+                "config": {"workload": CONFIGS["C5"][5], "fill_of_free_hbm": args.fill, "nrhs": 1,
+                           "parallelism": f"batch-shard x{world}", "l2": "inputs larger than L2 (>= 1 GB per point)"},
+                "hbm_gbs": tot_bytes / (tot_ms * 1e-3) / 1e9,
+                "roofline": {"kernel": "whole step (sweep aggregate)", "bound": "hbm",
+                             "achieved": tot_bytes / (tot_ms * 1e-3) / 1e9, "peak": peak, "unit": "GB/s",
+                             "frac": tot_bytes / (tot_ms * 1e-3) / 1e9 / peak, "peak_kind": peak_kind,
+                             "traffic": None, "best_point": {k: best[k] for k in ("n", "kl", "ku", "hbm_gbs")}},
+                "e2e": None, "gpu_launches": 2 * args.steps * len(points), "clocks": clocks, "sweep": points}
+        print(json.dumps(line))
+    if world > 1:
+        dist.destroy_process_group()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -146,8 +247,15 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--fill", type=float, default=0.2, help="C5: fraction of free HBM per sweep point")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
+    if args.config == "C5":
+        if args.impl == "reference":
+            print(json.dumps({"impl": "reference", "unavailable": "C5 reference arm not run (use a fixed config)"}))
+            return
+        run_sweep(args, int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1")))
+        return
 
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -241,7 +349,8 @@ def main():
     glob = bpg * world
     value = glob * (f_trf + f_trs) / (ms_step * 1e-3) / 1e9
     hbm = glob * (b_trf + b_trs) / (ms_step * 1e-3) / 1e9  # SURVEY 8(d) bytes of trf + trs
-    fused = nrhs == 1 and bl.trf_variant(n, n, kl, ku) == bl.WINDOW
+    v_trf = bl.trf_variant(n, n, kl, ku)
+    fused = nrhs == 1 and v_trf in (bl.WINDOW, bl.ROWS)  # dgbtrfs fuses the forward solve (run_trfs)
     k_trf, k_trs = (fb_trf, fb_trs) if fused else (b_trf, b_trs)  # bytes each launch of THIS path moves
     hbm_moved = glob * (k_trf + k_trs) / (ms_step * 1e-3) / 1e9
 
@@ -275,7 +384,9 @@ def main():
         return
 
     peak, peak_kind = peaks()
-    dom = "gbtrf_window_kernel" if trf_ms >= trs_ms else "gbtrs_window_kernel"
+    trf_kernel = {bl.ROWS: "gbtrf_rows_kernel", bl.WINDOW: "gbtrf_window_kernel"}.get(v_trf, "gbtrf_generic_kernel")
+    trs_kernel = "gbtrs_window_kernel" if bl.trs_variant(n, kl, ku, nrhs) == bl.WINDOW else "gbtrs_generic_kernel"
+    dom = trf_kernel if trf_ms >= trs_ms else trs_kernel
     dom_ms = (trf_ms if trf_ms >= trs_ms else trs_ms) / args.steps
     dom_bytes = cnt * (k_trf if trf_ms >= trs_ms else k_trs)
     achieved = dom_bytes / (dom_ms * 1e-3) / 1e9

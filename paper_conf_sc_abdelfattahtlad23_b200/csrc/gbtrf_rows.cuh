@@ -57,7 +57,10 @@ struct TrfRows {
     static constexpr int BIT = (BK * U + G - 1) / G;
     static_assert(BIT <= 32, "block element mask");
     static constexpr int WARPS_FIT = (72 * 1024) / (GPW * GROUP_DBL * 8);
-    static constexpr int WARPS = WARPS_FIT < 1 ? 1 : (WARPS_FIT < BANDLU_ROWS_WARPS ? WARPS_FIT : BANDLU_ROWS_WARPS);
+    // wide windows (W > 24) run 8 warps/SM: 2 per scheduler, so each thread may use up to 255
+    // registers (the register file is split per scheduler: 3 warps each would cap it at 168)
+    static constexpr int WMAX = W > 24 ? 2 : BANDLU_ROWS_WARPS;
+    static constexpr int WARPS = WARPS_FIT < 1 ? 1 : (WARPS_FIT < WMAX ? WARPS_FIT : WMAX);
 #ifndef BANDLU_ROWS_MINW
 #define BANDLU_ROWS_MINW 12
 #endif

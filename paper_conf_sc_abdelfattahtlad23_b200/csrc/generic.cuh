@@ -79,12 +79,19 @@ __global__ void __launch_bounds__(128) gbtrf_generic_kernel(int m, int n, int kl
                 const double rcp = 1.0 / AB(kv, j);
                 for (int i = 1 + lane; i <= km; i += 32) AB(kv + i, j) = AB(kv + i, j) * rcp;
                 __syncwarp();
+                // lanes over rows i (multiplier in a register), loop over columns c:
+                // U(j, j+c) is one broadcast load, rows i of column j+c are contiguous
                 const int w = ju - j;
-                const int tot = w * km;
-                for (int e = lane; e < tot; e += 32) {
-                    const int c = 1 + e / km, i = 1 + e % km;
-                    const double y = AB(kv - c, j + c);
-                    if (y != 0.0) AB(kv + i - c, j + c) = __fma_rn(AB(kv + i, j), -y, AB(kv + i - c, j + c));
+                for (int i0 = 1; i0 <= km; i0 += 32) {
+                    const int i = i0 + lane;
+                    const bool row = i <= km;
+                    const double l = row ? AB(kv + i, j) : 0.0;
+                    double *a = &AB(kv + i - 1, j + 1);  // AB(kv+i-c, j+c) for c = 1
+#pragma unroll 4
+                    for (int c = 1; c <= w; ++c, a += ldab - 1) {
+                        const double y = AB(kv - c, j + c);
+                        if (y != 0.0 && row) *a = __fma_rn(l, -y, *a);
+                    }
                 }
                 __syncwarp();
             }

@@ -15,6 +15,8 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 OUT = os.path.join(ROOT, "gpurun_out")
 PROF = os.path.join(ROOT, "profiles")
 
+KERNELS = ("gbtrf_rows_kernel", "gbtrf_window_kernel", "gbtrf_tc_kernel", "gbtrf_generic_kernel",
+           "gbtrs_window_kernel", "gbtrs_generic_kernel", "gbtrs_t_generic_kernel")
 KEYS = {
     "duration_us": ("gpu__time_duration.sum", 1e-3),
     "dram_bytes_read": ("dram__bytes_read.sum", 1.0),
@@ -43,7 +45,7 @@ def summarise(rep):
     out = {}
     for row in rows:
         name = row[hdr.index("Kernel Name")]
-        kern = "gbtrf_window_kernel" if "gbtrf" in name else ("gbtrs_window_kernel" if "gbtrs" in name else name)
+        kern = next((k for k in KERNELS if k in name), name)
         d = {"kernel_full": name}
         for k, (m, _) in KEYS.items():
             if m in hdr:
@@ -80,7 +82,7 @@ def launches(csvpath):
     agg = {}
     for row in r:
         nm = row.get("Kernel Name", "")
-        key = "gbtrf_window_kernel" if "gbtrf_window" in nm else ("gbtrs_window_kernel" if "gbtrs_window" in nm else nm[:60])
+        key = next((k for k in KERNELS if k in nm), nm[:60])
         try:
             v = float(row["Metric Value"])
         except (KeyError, ValueError):
