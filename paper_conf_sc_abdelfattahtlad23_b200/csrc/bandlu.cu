@@ -12,6 +12,7 @@
 #include "../../include/bandlu.h"
 #include "common.cuh"
 #include "gbtrf_rows.cuh"
+#include "gbtrf_wide.cuh"
 #include "gbtrf_tc.cuh"
 #include "gbtrf_window.cuh"
 #include "gbtrs_window.cuh"
@@ -74,6 +75,17 @@ namespace {
     X(2, 32, 8, 1)
 #endif
 
+// (KL, KU) with kl+1 > 32: two-warp row-slot kernel (gbtrf_wide.cuh), dispatched as
+// BANDLU_ROWS; the solve uses the window trs kernel (BANDLU_TRS_LIST).
+#if defined(BANDLU_NO_ROWS) || defined(BANDLU_ONLY_C3)
+#define BANDLU_WIDE_LIST(X)
+#else
+#define BANDLU_WIDE_LIST(X) X(32, 32)
+#endif
+#define BANDLU_TRS_LIST(X) \
+    BANDLU_WINDOW_LIST(X)  \
+    BANDLU_WIDE_LIST(X)
+
 // trs launch geometry: target resident warps (148 SMs x 8)
 #ifndef BANDLU_TRS_WPSM
 #define BANDLU_TRS_WPSM 8
@@ -116,6 +128,16 @@ int launch_trf_rows(int m, int n, AP A, int ldab, PP P, int *info, int batch, cu
     return cuda_ret(cudaGetLastError());
 }
 
+template <int KL, int KU, bool FWD, class AP, class PP, class BP>
+int launch_trf_wide(int m, int n, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st, BP B) {
+    using C = TrfWide<KL, KU>;
+    auto k = gbtrf_wide_kernel<KL, KU, FWD, AP, PP, BP>;
+    size_t sm = C::smem_bytes();
+    if (int r = set_smem(k, sm)) return r;
+    k<<<(unsigned)batch, 64, sm, st>>>(m, n, A, ldab, P, info, batch, B);
+    return cuda_ret(cudaGetLastError());
+}
+
 template <class AP, class PP>
 int launch_trf_generic(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st) {
     const unsigned grid = (unsigned)(((int64_t)batch * 32 + 127) / 128);
@@ -131,10 +153,26 @@ bool trf_window_available(int kl, int ku) {
     return false;
 }
 
+bool trf_wide_available(int kl, int ku) {
+#define X(a, b) \
+    if (kl == a && ku == b) return true;
+    BANDLU_WIDE_LIST(X)
+#undef X
+    return false;
+}
+
 bool trf_rows_available(int kl, int ku) {
 #define X(a, b, g, r) \
     if (kl == a && ku == b) return true;
     BANDLU_ROWS_LIST(X)
+#undef X
+    return trf_wide_available(kl, ku);
+}
+
+bool trs_window_available(int kl, int ku) {
+#define X(a, b) \
+    if (kl == a && ku == b) return true;
+    BANDLU_TRS_LIST(X)
 #undef X
     return false;
 }
@@ -181,6 +219,10 @@ int run_trf(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int b
 #define X(a, b, g, r) \
     if (kl == a && ku == b) return launch_trf_rows<a, b, g, r, false>(m, n, A, ldab, P, info, batch, st, Strided<double>{nullptr, 0});
         BANDLU_ROWS_LIST(X)
+#undef X
+#define X(a, b) \
+    if (kl == a && ku == b) return launch_trf_wide<a, b, false>(m, n, A, ldab, P, info, batch, st, Strided<double>{nullptr, 0});
+        BANDLU_WIDE_LIST(X)
 #undef X
         return BANDLU_ERR_UNSUPPORTED;
     }
@@ -229,7 +271,7 @@ int launch_trs_generic(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP
 int pick_trs(int n, int kl, int ku, int nrhs) {
     (void)n;
     (void)nrhs;
-    return trf_window_available(kl, ku) ? BANDLU_WINDOW : BANDLU_GENERIC;
+    return trs_window_available(kl, ku) ? BANDLU_WINDOW : BANDLU_GENERIC;
 }
 
 template <class AP, class PP, class BP>
@@ -253,7 +295,7 @@ int run_trs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ldb
     if (variant == BANDLU_WINDOW) {
 #define X(a, b) \
     if (kl == a && ku == b) return launch_trs_window<a, b>(n, nrhs, A, ldab, P, B, ldb, skip, batch, st);
-        BANDLU_WINDOW_LIST(X)
+        BANDLU_TRS_LIST(X)
 #undef X
         return BANDLU_ERR_UNSUPPORTED;
     }
@@ -273,7 +315,7 @@ template <class AP, class PP, class BP>
 int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ldb, int *info, int batch,
              cudaStream_t st, int phase) {
     if (batch == 0) return 0;
-    if (n > 0 && nrhs == 1 && trf_window_available(kl, ku)) {
+    if (n > 0 && nrhs == 1 && (trf_window_available(kl, ku) || trf_wide_available(kl, ku))) {
         int r = BANDLU_ERR_UNSUPPORTED;
         Strided<const double> Ac{A.base, A.stride};
         Strided<const int> Pc{P.base, P.stride};
@@ -285,6 +327,14 @@ int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ld
         if (r == 0 && phase != 1) r = launch_trs_window<a, b>(n, 1, Ac, ldab, Pc, B, ldb, nullptr, batch, st, 0); \
     }
             BANDLU_ROWS_LIST(X)
+#undef X
+#define X(a, b)                                                                                           \
+    if (kl == a && ku == b) {                                                                             \
+        r = 0;                                                                                            \
+        if (phase != 2) r = launch_trf_wide<a, b, true>(n, n, A, ldab, P, info, batch, st, B);           \
+        if (r == 0 && phase != 1) r = launch_trs_window<a, b>(n, 1, Ac, ldab, Pc, B, ldb, nullptr, batch, st, 0); \
+    }
+            BANDLU_WIDE_LIST(X)
 #undef X
             return r;
         }

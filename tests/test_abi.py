@@ -112,7 +112,9 @@ def test_variant_heuristic_is_shape_only(lib):
     assert b.rows_available(10, 10) and b.rows_available(2, 32) and not b.rows_available(1, 1)
     assert b.tc_available(10, 10) and not b.tc_available(1, 1)  # opt-in tensor-core kernel
     assert b.trf_variant(256, 256, 1, 1) == b.WINDOW
-    assert b.trf_variant(100, 100, 32, 32) == b.GENERIC  # kl+1 > 32 lanes: safeguard kernel
+    assert b.trf_variant(100, 100, 32, 32) == b.ROWS  # kl+1 > 32 lanes: two-warp row-slot kernel
+    assert b.trf_variant(100, 100, 33, 20) == b.GENERIC  # band not compiled: safeguard kernel
+    assert b.trs_variant(100, 32, 32, 1) == b.WINDOW
     assert b.trf_variant(0, 5, 1, 1) == b.GENERIC
     assert b.trs_variant(1024, 2, 32, 16) == b.WINDOW
 

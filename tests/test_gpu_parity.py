@@ -22,6 +22,8 @@ pytestmark = pytest.mark.gpu
 import paper_conf_sc_abdelfattahtlad23_b200 as bl  # noqa: E402
 
 WINDOW_BANDS = [(0, 0), (0, 3), (1, 1), (2, 2), (2, 3), (3, 0), (3, 2), (4, 4), (10, 7), (10, 10), (2, 32)]
+WIDE_BANDS = [(32, 32)]  # kl+1 > 32: two-warp ROWS factorization, window solve kernel
+ALL_BANDS = WINDOW_BANDS + WIDE_BANDS
 
 
 def _gpu_trf(A_np, m, n, kl, ku, variant=bl.AUTO):
@@ -38,7 +40,7 @@ def trf_variants(kl, ku):
     """Forced factorization variants to cross-check: the safeguard, the row-owner
     window, and the row-slot (ROWS) and tensor-core (DMMA) kernels where they are
     compiled for (kl, ku)."""
-    v = [bl.WINDOW, bl.GENERIC]
+    v = [bl.WINDOW, bl.GENERIC] if (kl, ku) in WINDOW_BANDS else [bl.GENERIC]
     if bl.rows_available(kl, ku):
         v.append(bl.ROWS)
     if bl.tc_available(kl, ku):
@@ -58,7 +60,7 @@ def _check_trf(m, n, kl, ku, batch, variant, ldab=None, first=0, A_in=None):
     return Ao, ipo, info_o
 
 
-@pytest.mark.parametrize("kl,ku", WINDOW_BANDS)
+@pytest.mark.parametrize("kl,ku", ALL_BANDS)
 @pytest.mark.parametrize("variant", [bl.WINDOW, bl.GENERIC, bl.ROWS, bl.TC])
 @pytest.mark.parametrize("n", [1, 2, 7, 37, 100])
 def test_trf_parity_small(kl, ku, variant, n):
@@ -68,7 +70,7 @@ def test_trf_parity_small(kl, ku, variant, n):
     _check_trf(n, n, kl, ku, batch=37, variant=variant)
 
 
-@pytest.mark.parametrize("kl,ku", WINDOW_BANDS)
+@pytest.mark.parametrize("kl,ku", ALL_BANDS)
 @pytest.mark.parametrize("mn", [(30, 20), (20, 30), (5, 40), (40, 5), (1, 9), (9, 1)])
 def test_trf_parity_rectangular(kl, ku, mn):
     m, n = mn
@@ -82,14 +84,14 @@ def test_trf_parity_generic_any_band(kl, ku):
     assert bl.trf_variant(150, 150, kl, ku) in (bl.GENERIC, bl.WINDOW, bl.ROWS)
 
 
-@pytest.mark.parametrize("kl,ku", [(1, 1), (10, 10), (2, 32)])
+@pytest.mark.parametrize("kl,ku", [(1, 1), (10, 10), (2, 32), (32, 32)])
 def test_trf_parity_padded_ldab(kl, ku):
     ldab = 2 * kl + ku + 1 + 3  # extra NaN rows at the bottom stay untouched
     for variant in trf_variants(kl, ku):
         _check_trf(70, 70, kl, ku, batch=5, variant=variant, ldab=ldab)
 
 
-@pytest.mark.parametrize("kl,ku", [(1, 1), (2, 3), (10, 10), (2, 32), (0, 3), (3, 0)])
+@pytest.mark.parametrize("kl,ku", [(1, 1), (2, 3), (10, 10), (2, 32), (0, 3), (3, 0), (32, 32)])
 def test_trf_parity_planted_zero_pivots(kl, ku):
     n = 60
     A = I.gen_band(n, n, kl, ku, count=6)
@@ -103,7 +105,7 @@ def test_trf_parity_planted_zero_pivots(kl, ku):
         assert list(info) == [1, 2, 30, 59, 60, 11]
 
 
-@pytest.mark.parametrize("kl,ku", [(1, 1), (2, 2), (10, 10), (2, 32)])
+@pytest.mark.parametrize("kl,ku", [(1, 1), (2, 2), (10, 10), (2, 32), (32, 32)])
 def test_trf_parity_exact_ties(kl, ku):
     """Integer-valued bands with many exact |pivot| ties: both sides take the
     same decision (first index, Q2) in the same precision."""
@@ -123,7 +125,7 @@ def _gpu_trs(Af, ipiv, B_np, n, kl, ku, variant=bl.AUTO):
     return B.cpu().numpy()
 
 
-@pytest.mark.parametrize("kl,ku", WINDOW_BANDS)
+@pytest.mark.parametrize("kl,ku", ALL_BANDS)
 @pytest.mark.parametrize("nrhs", [1, 2, 3, 16, 33])
 @pytest.mark.parametrize("variant", [bl.WINDOW, bl.GENERIC])
 def test_trs_parity(kl, ku, nrhs, variant):
@@ -139,7 +141,7 @@ def test_trs_parity(kl, ku, nrhs, variant):
 
 
 @pytest.mark.parametrize("n", [1, 2, 3, 8, 9, 130])
-@pytest.mark.parametrize("kl,ku", [(1, 1), (10, 10), (2, 32), (0, 0)])
+@pytest.mark.parametrize("kl,ku", [(1, 1), (10, 10), (2, 32), (0, 0), (32, 32)])
 def test_trs_parity_sizes(n, kl, ku):
     A = I.gen_band(n, n, kl, ku, count=7)
     ipiv, info = oracle.dgbtrf(A, n, n, kl, ku)
@@ -351,7 +353,7 @@ def test_application_shaped_workloads(batch, n, kl, ku):
     assert np.all(same_bits(Bg.cpu().numpy(), Bo))
 
 
-@pytest.mark.parametrize("kl,ku", [(10, 10), (2, 32), (10, 7)])
+@pytest.mark.parametrize("kl,ku", [(10, 10), (2, 32), (10, 7), (32, 32)])
 def test_trf_batch_tail_after_other_launches(kl, ku):
     """Batch tails leave dead matrix groups in the last CTA; they must not act on
     shared memory left over by earlier launches (regression: a dead group once
