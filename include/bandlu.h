@@ -83,9 +83,12 @@ enum bandlu_variant {
     BANDLU_TC = 3,      /* dgbtrf only, opt-in: window in FP64 tensor-core (DMMA) fragments, compiled
                            (kl, ku) with kl+1 <= 16 (bandlu_tc_available); same LAPACK operation
                            sequence, bitwise equal results */
-    BANDLU_ROWS = 4     /* dgbtrf only: register window with R row slots per lane and block-preloaded
+    BANDLU_ROWS = 4     /* dgbtrf: register window with R row slots per lane and block-preloaded
                            band rows, compiled (kl, ku) only (bandlu_rows_available); AUTO prefers it
-                           where compiled; bitwise equal results */
+                           where compiled.  dgbtrs ('N'): one lane per RHS row, a group of
+                           pow2 >= kl+ku+1 lanes per (matrix, RHS column), compiled (kl, ku) with
+                           kl+ku+1 <= 32 only (bandlu_trs_rows_available); AUTO's choice for
+                           nrhs == 1 with kl+ku+1 <= 4.  Bitwise equal results */
 };
 
 /* ---- dgbtrf: band LU with partial pivoting ---- */
@@ -184,6 +187,8 @@ int bandlu_trs_variant(int n, int kl, int ku, int nrhs);
 int bandlu_tc_available(int kl, int ku);
 /* 1 if a row-slot (BANDLU_ROWS) factorization kernel is compiled for (kl, ku), else 0. */
 int bandlu_rows_available(int kl, int ku);
+/* 1 if a lane-per-row solve kernel (dgbtrs BANDLU_ROWS) is compiled for (kl, ku), else 0. */
+int bandlu_trs_rows_available(int kl, int ku);
 /* ABI version of this library. */
 int bandlu_version(void);
 

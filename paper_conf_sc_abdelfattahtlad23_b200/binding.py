@@ -69,6 +69,7 @@ def load(build_if_missing: bool = False):
         "bandlu_trf_variant": [i, i, i, i],
         "bandlu_tc_available": [i, i],
         "bandlu_rows_available": [i, i],
+        "bandlu_trs_rows_available": [i, i],
         "bandlu_trs_variant": [i, i, i, i],
         "bandlu_version": [],
     }
@@ -83,7 +84,7 @@ def load(build_if_missing: bool = False):
 # exported symbol list (checked by tests against include/bandlu.h)
 EXPORTS = ("dgbtrf_batched", "dgbtrf_strided_batched", "dgbtrf_strided_batched_ex", "dgbtrs_batched",
            "dgbtrs_strided_batched", "dgbtrs_strided_batched_ex", "dgbsv_batched", "dgbsv_strided_batched",
-           "dgbsv_strided_batched_host", "dgbtrfs_strided_batched", "dgbtrfs_strided_batched_ex", "bandlu_trf_variant", "bandlu_trs_variant", "bandlu_tc_available", "bandlu_rows_available",
+           "dgbsv_strided_batched_host", "dgbtrfs_strided_batched", "dgbtrfs_strided_batched_ex", "bandlu_trf_variant", "bandlu_trs_variant", "bandlu_tc_available", "bandlu_rows_available", "bandlu_trs_rows_available",
            "bandlu_version")
 
 
@@ -212,6 +213,11 @@ def tc_available(kl: int, ku: int) -> bool:
 def rows_available(kl: int, ku: int) -> bool:
     """True if a row-slot factorization kernel (variant ROWS) is compiled for (kl, ku)."""
     return bool(load().bandlu_rows_available(kl, ku))
+
+
+def trs_rows_available(kl: int, ku: int) -> bool:
+    """True if a lane-per-row solve kernel (dgbtrs variant ROWS) is compiled for (kl, ku)."""
+    return bool(load().bandlu_trs_rows_available(kl, ku))
 
 
 def trs_variant(n: int, kl: int, ku: int, nrhs: int) -> int:

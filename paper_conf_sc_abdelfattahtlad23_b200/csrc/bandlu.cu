@@ -15,6 +15,7 @@
 #include "gbtrf_wide.cuh"
 #include "gbtrf_tc.cuh"
 #include "gbtrf_window.cuh"
+#include "gbtrs_rows.cuh"
 #include "gbtrs_window.cuh"
 #include "generic.cuh"
 
@@ -85,6 +86,25 @@ namespace {
 #define BANDLU_TRS_LIST(X) \
     BANDLU_WINDOW_LIST(X)  \
     BANDLU_WIDE_LIST(X)
+// (KL, KU) with kl+ku+1 <= 32 compiled as lane-per-row solve kernels
+// (gbtrs_rows.cuh); AUTO's choice for nrhs == 1.
+#ifdef BANDLU_ONLY_C3
+#define BANDLU_TRS_ROWS_LIST(X) \
+    X(1, 1)                     \
+    X(10, 10)
+#else
+#define BANDLU_TRS_ROWS_LIST(X) \
+    X(0, 0)                     \
+    X(0, 3)                     \
+    X(1, 1)                     \
+    X(2, 2)                     \
+    X(2, 3)                     \
+    X(3, 0)                     \
+    X(3, 2)                     \
+    X(4, 4)                     \
+    X(10, 7)                    \
+    X(10, 10)
+#endif
 
 // trs launch geometry: target resident warps (148 SMs x 8)
 #ifndef BANDLU_TRS_WPSM
@@ -177,6 +197,14 @@ bool trs_window_available(int kl, int ku) {
     return false;
 }
 
+bool trs_rows_available(int kl, int ku) {
+#define X(a, b) \
+    if (kl == a && ku == b) return true;
+    BANDLU_TRS_ROWS_LIST(X)
+#undef X
+    return false;
+}
+
 bool trf_tc_available(int kl, int ku) {
 #define X(a, b) \
     if (kl == a && ku == b) return true;
@@ -259,6 +287,17 @@ int launch_trs_window(int n, int nrhs, AP A, int ldab, PP P, BP B, int ldb, cons
     return cuda_ret(cudaGetLastError());
 }
 
+template <int KL, int KU, class AP, class PP, class BP>
+int launch_trs_rows(int n, int nrhs, AP A, int ldab, PP P, BP B, int ldb, const int *skip, int batch,
+                    cudaStream_t st, int fwd = 1) {
+    using C = TrsRows<KL, KU>;
+    auto k = fwd ? gbtrs_rows_kernel<KL, KU, true, AP, PP, BP> : gbtrs_rows_kernel<KL, KU, false, AP, PP, BP>;
+    const int64_t units = (int64_t)batch * nrhs, per_block = (int64_t)C::WARPS * C::GPW;
+    const unsigned grid = (unsigned)((units + per_block - 1) / per_block);
+    k<<<grid, C::WARPS * 32, 0, st>>>(n, nrhs, A, ldab, P, B, ldb, skip, batch);
+    return cuda_ret(cudaGetLastError());
+}
+
 template <class AP, class PP, class BP>
 int launch_trs_generic(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ldb, const int *skip,
                        int batch, cudaStream_t st) {
@@ -268,9 +307,15 @@ int launch_trs_generic(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP
     return cuda_ret(cudaGetLastError());
 }
 
+// The lane-per-row solve issues one division and one broadcast per matrix-step
+// (the window solve one per 32/R matrices); it only wins where a warp packs
+// >= 8 matrices (kl+ku+1 <= 4): measured C2 (1,1) 0.097 vs 0.105 ms, but C3
+// (10,10) 0.78 vs 0.32 ms and PELE-like (10,10) 0.083 vs 0.039 ms.
+bool trs_rows_preferred(int kl, int ku) { return kl + ku + 1 <= 4 && trs_rows_available(kl, ku); }
+
 int pick_trs(int n, int kl, int ku, int nrhs) {
     (void)n;
-    (void)nrhs;
+    if (nrhs == 1 && trs_rows_preferred(kl, ku)) return BANDLU_ROWS;
     return trs_window_available(kl, ku) ? BANDLU_WINDOW : BANDLU_GENERIC;
 }
 
@@ -299,8 +344,26 @@ int run_trs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ldb
 #undef X
         return BANDLU_ERR_UNSUPPORTED;
     }
+    if (variant == BANDLU_ROWS) {
+#define X(a, b) \
+    if (kl == a && ku == b) return launch_trs_rows<a, b>(n, nrhs, A, ldab, P, B, ldb, skip, batch, st);
+        BANDLU_TRS_ROWS_LIST(X)
+#undef X
+        return BANDLU_ERR_UNSUPPORTED;
+    }
     if (variant != BANDLU_GENERIC) return BANDLU_ERR_UNSUPPORTED;
     return launch_trs_generic(n, kl, ku, nrhs, A, ldab, P, B, ldb, skip, batch, st);
+}
+
+// backward-only solve after the fused factorization (nrhs == 1)
+template <int KL, int KU, class AP, class PP, class BP>
+int launch_trs_bwd(int n, AP A, int ldab, PP P, BP B, int ldb, int batch, cudaStream_t st) {
+#ifndef BANDLU_TRS_BWD_WINDOW
+    if constexpr (KL + KU + 1 <= 32) {
+        if (trs_rows_preferred(KL, KU)) return launch_trs_rows<KL, KU>(n, 1, A, ldab, P, B, ldb, nullptr, batch, st, 0);
+    }
+#endif
+    return launch_trs_window<KL, KU>(n, 1, A, ldab, P, B, ldb, nullptr, batch, st, 0);
 }
 
 // ------------------------------------- fused factor + solve (dgbtrf; dgbtrs)
@@ -324,7 +387,7 @@ int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ld
     if (kl == a && ku == b) {                                                                             \
         r = 0;                                                                                            \
         if (phase != 2) r = launch_trf_rows<a, b, g, rr, true>(n, n, A, ldab, P, info, batch, st, B);     \
-        if (r == 0 && phase != 1) r = launch_trs_window<a, b>(n, 1, Ac, ldab, Pc, B, ldb, nullptr, batch, st, 0); \
+        if (r == 0 && phase != 1) r = launch_trs_bwd<a, b>(n, Ac, ldab, Pc, B, ldb, batch, st); \
     }
             BANDLU_ROWS_LIST(X)
 #undef X
@@ -332,7 +395,7 @@ int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ld
     if (kl == a && ku == b) {                                                                             \
         r = 0;                                                                                            \
         if (phase != 2) r = launch_trf_wide<a, b, true>(n, n, A, ldab, P, info, batch, st, B);           \
-        if (r == 0 && phase != 1) r = launch_trs_window<a, b>(n, 1, Ac, ldab, Pc, B, ldb, nullptr, batch, st, 0); \
+        if (r == 0 && phase != 1) r = launch_trs_bwd<a, b>(n, Ac, ldab, Pc, B, ldb, batch, st); \
     }
             BANDLU_WIDE_LIST(X)
 #undef X
@@ -342,7 +405,7 @@ int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ld
     if (kl == a && ku == b) {                                                                             \
         r = 0;                                                                                            \
         if (phase != 2) r = launch_trf_window<a, b, true>(n, n, A, ldab, P, info, batch, st, B);          \
-        if (r == 0 && phase != 1) r = launch_trs_window<a, b>(n, 1, Ac, ldab, Pc, B, ldb, nullptr, batch, st, 0); \
+        if (r == 0 && phase != 1) r = launch_trs_bwd<a, b>(n, Ac, ldab, Pc, B, ldb, batch, st); \
     }
         BANDLU_WINDOW_LIST(X)
 #undef X
@@ -424,6 +487,7 @@ int bandlu_version(void) { return 1; }
 int bandlu_trf_variant(int m, int n, int kl, int ku) { return pick_trf(m, n, kl, ku); }
 int bandlu_tc_available(int kl, int ku) { return trf_tc_available(kl, ku) ? 1 : 0; }
 int bandlu_rows_available(int kl, int ku) { return trf_rows_available(kl, ku) ? 1 : 0; }
+int bandlu_trs_rows_available(int kl, int ku) { return trs_rows_available(kl, ku) ? 1 : 0; }
 int bandlu_trs_variant(int n, int kl, int ku, int nrhs) { return pick_trs(n, kl, ku, nrhs); }
 
 int dgbtrf_strided_batched_ex(int m, int n, int kl, int ku, double *dA, int ldab, int64_t strideA, int *dipiv,

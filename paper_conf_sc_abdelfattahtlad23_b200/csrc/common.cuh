@@ -150,6 +150,20 @@ __device__ __forceinline__ uint64_t abs_key(double x) {
     return static_cast<uint64_t>(__double_as_longlong(x)) & 0x7fffffffffffffffull;
 }
 
+// RN(a / b) on lanes where p holds, else a.  The compiler if-converts a
+// guarded division and runs it on every lane; lanes with !p divide 1 by 1 so
+// that none of them leaves the inline fast path for the slow-path CALL (0 / 0
+// would), and a CALL waits for every outstanding load of the warp.
+// The operands pass through an opaque move: otherwise the compiler sees that
+// q is only used where p holds and divides a by b on every lane again.
+__device__ __forceinline__ double ddiv_rn_if(bool p, double a, double b) {
+    double na, nb;
+    asm("mov.b64 %0, %1;" : "=d"(na) : "d"(p ? a : 1.0));
+    asm("mov.b64 %0, %1;" : "=d"(nb) : "d"(p ? b : 1.0));
+    const double q = __ddiv_rn(na, nb);
+    return p ? q : a;
+}
+
 __host__ __device__ constexpr int pow2_ceil(int x) {
     int p = 1;
     while (p < x) p *= 2;

@@ -137,15 +137,33 @@ __global__ void __launch_bounds__(TrfRows<KL, KU, G, R>::WARPS * 32, TrfRows<KL,
         const int e = t + k * G, bs = e % U, bk = e / U;
         if (bk < BK && bk - bs >= 0 && bk - bs <= KV) bmask |= 1u << k;
     }
+    // G % U == 0: lane t always moves row offset bs = t % U of the block, columns
+    // bk = t / U + k * KS -- per-k offsets are immediates / one pointer stride
+    constexpr int KS = G / U;
+    const int64_t kstride = (int64_t)KS * (ldab - 1);
     auto stage_block = [&](int qb, const double *colq) {
+        if constexpr (G % U == 0) {
+            const int q = qb + t % U, c0 = qb - KL + t / U;
+            const bool rowok = q < mloc;
+            const uint32_t dst0 = ring_s + (uint32_t)(((q & (RR - 1)) * WP + 1 + t / U) * 8);
+            const double *src = colq + bo0 + (KV + KL);
 #pragma unroll
-        for (int k = 0; k < BIT; ++k) {
-            const int e = t + k * G, bs = e % U, bk = e / U;
-            if (bmask >> k & 1u) {
-                const int q = qb + bs;
-                const bool ok = (q < mloc) && (qb - KL + bk < n);
-                const uint32_t dst = ring_s + (uint32_t)(((q & (RR - 1)) * WP + 1 + bk) * 8);
-                cp_async8(dst, ok ? colq + boff(k) + (KV + KL) : safe, ok ? 8u : 0u);
+            for (int k = 0; k < BIT; ++k) {
+                if (bmask >> k & 1u) {
+                    const bool ok = rowok && (c0 + k * KS < n);
+                    cp_async8(dst0 + (uint32_t)(k * KS * 8), ok ? src + k * kstride : safe, ok ? 8u : 0u);
+                }
+            }
+        } else {
+#pragma unroll
+            for (int k = 0; k < BIT; ++k) {
+                const int e = t + k * G, bs = e % U, bk = e / U;
+                if (bmask >> k & 1u) {
+                    const int q = qb + bs;
+                    const bool ok = (q < mloc) && (qb - KL + bk < n);
+                    const uint32_t dst = ring_s + (uint32_t)(((q & (RR - 1)) * WP + 1 + bk) * 8);
+                    cp_async8(dst, ok ? colq + boff(k) + (KV + KL) : safe, ok ? 8u : 0u);
+                }
             }
         }
         if constexpr (FWD) {
@@ -316,11 +334,23 @@ __global__ void __launch_bounds__(TrfRows<KL, KU, G, R>::WARPS * 32, TrfRows<KL,
         }
         // ---- U rows j0 .. j0+U-1 (the block's records) -> HBM, 32-byte column chunks
         __syncwarp();
+        if constexpr (G % U == 0) {
+            const bool rowok = live && j0 + t % U < mn;
+            const int c0 = j0 + t / U;
+            const uint32_t src0 = rec_s + (uint32_t)(((t % U) * WP + t / U) * 8);
+            double *dst = colb + bo0 + KV;
 #pragma unroll
-        for (int k = 0; k < BIT; ++k) {
-            const int e = t + k * G, bs = e % U, bk = e / U;
-            if (live && (bmask >> k & 1u) && j0 + bs < mn && j0 + bk < n)
-                colb[boff(k) + KV] = ld_shared_f64(rec_s + (uint32_t)((bs * WP + bk) * 8));
+            for (int k = 0; k < BIT; ++k) {
+                if ((bmask >> k & 1u) && rowok && c0 + k * KS < n)
+                    dst[k * kstride] = ld_shared_f64(src0 + (uint32_t)(k * KS * 8));
+            }
+        } else {
+#pragma unroll
+            for (int k = 0; k < BIT; ++k) {
+                const int e = t + k * G, bs = e % U, bk = e / U;
+                if (live && (bmask >> k & 1u) && j0 + bs < mn && j0 + bk < n)
+                    colb[boff(k) + KV] = ld_shared_f64(rec_s + (uint32_t)((bs * WP + bk) * 8));
+            }
         }
         colb += (int64_t)U * ldab;
         __syncwarp();

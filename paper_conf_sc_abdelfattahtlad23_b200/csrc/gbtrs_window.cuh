@@ -40,6 +40,10 @@
 #define BANDLU_TRS_NS_NARROW 16
 #endif
 
+#ifndef BANDLU_TRS_NS_WIDE
+#define BANDLU_TRS_NS_WIDE 8
+#endif
+
 namespace bandlu {
 
 template <int KL_, int KU_>
@@ -47,7 +51,7 @@ struct TrsWin {
     static constexpr int KL = KL_, KU = KU_, KV = KL + KU;
     static constexpr int WF = KL + 1, WB = KV + 1;         // forward / backward window lengths
     // ring depth (column steps in flight): narrow bands need more steps to cover HBM latency
-    static constexpr int NS = (WB <= 5) ? BANDLU_TRS_NS_NARROW : 8;
+    static constexpr int NS = (WB <= 5) ? BANDLU_TRS_NS_NARROW : BANDLU_TRS_NS_WIDE;
     static constexpr int FMAX = (KL > WB ? KL : WB) + 2;   // factor doubles per slot (+16 B rounding)
     static constexpr int SP = (FMAX + 1) & ~1;             // even -> 16 B aligned slots
     // slot: [SP factor doubles][ipiv int, pad][R rhs doubles when rows move one per step]

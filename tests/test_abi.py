@@ -117,6 +117,10 @@ def test_variant_heuristic_is_shape_only(lib):
     assert b.trs_variant(100, 32, 32, 1) == b.WINDOW
     assert b.trf_variant(0, 5, 1, 1) == b.GENERIC
     assert b.trs_variant(1024, 2, 32, 16) == b.WINDOW
+    assert b.trs_variant(512, 10, 10, 1) == b.WINDOW  # lane-per-row solve measured slower here
+    assert b.trs_variant(256, 1, 1, 1) == b.ROWS  # nrhs = 1, kl+ku+1 <= 4: lane-per-row solve
+    assert b.trs_variant(512, 10, 10, 2) == b.WINDOW
+    assert b.trs_rows_available(1, 1) and not b.trs_rows_available(2, 32)
 
 
 def test_product_package_does_not_import_oracle():

@@ -127,8 +127,10 @@ def _gpu_trs(Af, ipiv, B_np, n, kl, ku, variant=bl.AUTO):
 
 @pytest.mark.parametrize("kl,ku", ALL_BANDS)
 @pytest.mark.parametrize("nrhs", [1, 2, 3, 16, 33])
-@pytest.mark.parametrize("variant", [bl.WINDOW, bl.GENERIC])
+@pytest.mark.parametrize("variant", [bl.WINDOW, bl.GENERIC, bl.ROWS])
 def test_trs_parity(kl, ku, nrhs, variant):
+    if variant == bl.ROWS and not bl.trs_rows_available(kl, ku):
+        pytest.skip("no lane-per-row solve kernel for this band")
     n, batch = 45, 13
     A = I.gen_band(n, n, kl, ku, count=batch)
     ipiv, info = oracle.dgbtrf(A, n, n, kl, ku)
@@ -148,7 +150,7 @@ def test_trs_parity_sizes(n, kl, ku):
     B = I.gen_rhs(n, 2, count=7)
     Bo = B.copy()
     oracle.dgbtrs(A, ipiv, Bo, n, kl, ku)
-    for variant in (bl.WINDOW, bl.GENERIC):
+    for variant in (bl.WINDOW, bl.GENERIC) + ((bl.ROWS,) if bl.trs_rows_available(kl, ku) else ()):
         assert np.all(same_bits(_gpu_trs(A, ipiv, B.copy(), n, kl, ku, variant), Bo))
 
 
