@@ -39,14 +39,17 @@ template <int KL_, int KU_, int G_, int R_>
 struct TrfRows {
     static constexpr int KL = KL_, KU = KU_, KV = KL + KU, W = KV + 1;
     static constexpr int G = G_, R = R_, GPW = 32 / G;
-    static constexpr int U = 4;                  // columns per block (window shift granularity)
+#ifndef BANDLU_ROWS_U
+#define BANDLU_ROWS_U 4
+#endif
+    static constexpr int U = BANDLU_ROWS_U;      // columns per block (window shift granularity)
     static constexpr int WS = W + U, H = (WS + 1) / 2;
     static_assert(G * R >= KL + 1 + U, "slots: KL+1 active rows + U preloaded rows");
     static_assert(32 % G == 0, "group size");
     // ring row / record pitch (doubles), spare pair at RP: (B entry[, logical row])
     static constexpr int WP = (G >= 8) ? ((2 * H + 2 + 11) / 16) * 16 + 4 : 2 * H + 2 + ((2 * H + 2) % 4 == 2 ? 0 : 2);
     static constexpr int RP = WP - 2;
-    static constexpr int D = 4, DB = D / U;      // staging lead (rows / blocks)
+    static constexpr int D = U, DB = D / U;      // staging lead (rows / blocks)
     static constexpr int RR = pow2_ceil((DB + 1) * U);
     static constexpr int NREC = U;
     // group pitch == 2 (mod 16) doubles: the GPW groups of a warp read their
@@ -91,8 +94,14 @@ __device__ __forceinline__ unsigned group_min_u32(unsigned v) {
     return v;
 }
 
+// BANDLU_ROWS_MAXREG (experiments): a register cap instead of the resident-CTA target
+#ifdef BANDLU_ROWS_MAXREG
+#define BANDLU_ROWS_BOUNDS(...) __maxnreg__(BANDLU_ROWS_MAXREG)
+#else
+#define BANDLU_ROWS_BOUNDS(...) __launch_bounds__(__VA_ARGS__::WARPS * 32, __VA_ARGS__::MINB)
+#endif
 template <int KL, int KU, int G, int R, bool FWD, class AP, class PP, class BP>
-__global__ void __launch_bounds__(TrfRows<KL, KU, G, R>::WARPS * 32, TrfRows<KL, KU, G, R>::MINB)
+__global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
     gbtrf_rows_kernel(int m, int n, AP A, int ldab, PP P, int *__restrict__ info, int batch, BP Bv) {
     using C = TrfRows<KL, KU, G, R>;
     constexpr int KV = C::KV, U = C::U, H = C::H, WP = C::WP, RP = C::RP, D = C::D, RR = C::RR, BK = C::BK,
@@ -289,7 +298,15 @@ __global__ void __launch_bounds__(TrfRows<KL, KU, G, R>::WARPS * 32, TrfRows<KL,
             // ---- broadcast read (64-bit: one cycle per warp for all groups)
             const double2 yp = ld_shared_v2(rcs + RP * 8);
             const int ppos = (int)__double_as_longlong(yp.y);
+#ifdef BANDLU_ROWS_SHFL_P
+            // pivot value straight from the pivot lane (off the record write -> read chain)
+            double xpv = x[0];
+#pragma unroll
+            for (int ri = 1; ri < R; ++ri) xpv = (rb == ri) ? x[ri] : xpv;
+            const double p = __shfl_sync(0xffffffffu, xpv, (int)gbase + max(__ffs(gb) - 1, 0));
+#else
             const double p = ld_volatile_shared_f64(rcs + s * 8);
+#endif
             const bool zp = (p == 0.0);
             if (is_piv) *ipj = ppos + 1;
             if (live && zp && linfo == 0) linfo = j + 1;
@@ -320,12 +337,27 @@ __global__ void __launch_bounds__(TrfRows<KL, KU, G, R>::WARPS * 32, TrfRows<KL,
                 }
             }
             // ---- RANK-1 update of the window columns j+1..j+KV (DGER, alpha = -1, FMA)
+#ifndef BANDLU_ROWS_LDS64
+            // 128-bit broadcast reads of slot pairs (2h, 2h+1) covering s+1 .. s+KV: half the
+            // load instructions of 64-bit reads for the same shared-memory wavefronts (C3
+            // factorization 1.016 -> 0.981 ms)
+#pragma unroll
+            for (int h = (s + 1) / 2; h <= (s + KV) / 2; ++h) {
+                const double2 u2 = ld_shared_v2(rcs + h * 16);
+#pragma unroll
+                for (int ri = 0; ri < R; ++ri) {
+                    if (2 * h >= s + 1) VS(ri, 2 * h) = __fma_rn(lu[ri], -u2.x, VS(ri, 2 * h));
+                    if (2 * h + 1 <= s + KV) VS(ri, 2 * h + 1) = __fma_rn(lu[ri], -u2.y, VS(ri, 2 * h + 1));
+                }
+            }
+#else
 #pragma unroll
             for (int k = 1; k <= KV; ++k) {
                 const double uk = ld_volatile_shared_f64(rcs + (s + k) * 8);
 #pragma unroll
                 for (int ri = 0; ri < R; ++ri) VS(ri, s + k) = __fma_rn(lu[ri], -uk, VS(ri, s + k));
             }
+#endif
 #pragma unroll
             for (int ri = 0; ri < R; ++ri)
                 if (pslot[ri]) pos[ri] = FREE;
@@ -358,14 +390,7 @@ __global__ void __launch_bounds__(TrfRows<KL, KU, G, R>::WARPS * 32, TrfRows<KL,
 #pragma unroll
         for (int ri = 0; ri < R; ++ri) {
 #pragma unroll
-            for (int h = 0; h < H; ++h) {
-                if (h + U / 2 < H) {
-                    v[ri][h] = v[ri][h + U / 2];
-                } else {
-                    v[ri][h].x = 0.0;
-                    v[ri][h].y = 0.0;
-                }
-            }
+            for (int k = 0; k < 2 * H; ++k) VS(ri, k) = (k + U < 2 * H) ? VS(ri, k + U) : 0.0;
         }
     }
     cp_async_wait<0>();
