@@ -5,8 +5,11 @@
 // host synchronisation on the device entry points.
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cstdint>
+#include <type_traits>
 #include <cstdio>
+#include <cstdlib>
 #include <mutex>
 
 #include "../../include/bandlu.h"
@@ -15,6 +18,7 @@
 #include "gbtrf_wide.cuh"
 #include "gbtrf_tc.cuh"
 #include "gbtrf_window.cuh"
+#include "gbtrs_bwd.cuh"
 #include "gbtrs_rows.cuh"
 #include "gbtrs_window.cuh"
 #include "generic.cuh"
@@ -355,6 +359,29 @@ int run_trs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ldb
     return launch_trs_generic(n, kl, ku, nrhs, A, ldab, P, B, ldb, skip, batch, st);
 }
 
+// lean backward-only solve (gbtrs_bwd.cuh); matrices per warp as the window solve
+template <int KL, int KU, class AP, class BP>
+int launch_trs_bwd_lean(int n, AP A, int ldab, BP B, int batch, cudaStream_t st) {
+    using C = TrsBwd<KL, KU>;
+    int gpw = 32;
+    while (gpw > 1 && batch < (int64_t)gpw * kTrsWarpsTarget) gpw >>= 1;
+    gpw = gpw < 2 ? 2 : gpw;
+    const size_t sm = C::smem_bytes(gpw);
+    const unsigned grid = (unsigned)((batch + gpw - 1) / gpw);
+    auto go = [&](auto k) -> int {
+        if (int r = set_smem(k, sm)) return r;
+        k<<<grid, 32, sm, st>>>(n, A, ldab, B, batch);
+        return cuda_ret(cudaGetLastError());
+    };
+    switch (gpw) {
+        case 2: return go(gbtrs_bwd_kernel<KL, KU, 2, AP, BP>);
+        case 4: return go(gbtrs_bwd_kernel<KL, KU, 4, AP, BP>);
+        case 8: return go(gbtrs_bwd_kernel<KL, KU, 8, AP, BP>);
+        case 16: return go(gbtrs_bwd_kernel<KL, KU, 16, AP, BP>);
+        default: return go(gbtrs_bwd_kernel<KL, KU, 32, AP, BP>);
+    }
+}
+
 // backward-only solve after the fused factorization (nrhs == 1)
 template <int KL, int KU, class AP, class PP, class BP>
 int launch_trs_bwd(int n, AP A, int ldab, PP P, BP B, int ldb, int batch, cudaStream_t st) {
@@ -362,6 +389,10 @@ int launch_trs_bwd(int n, AP A, int ldab, PP P, BP B, int ldb, int batch, cudaSt
     if constexpr (KL + KU + 1 <= 32) {
         if (trs_rows_preferred(KL, KU)) return launch_trs_rows<KL, KU>(n, 1, A, ldab, P, B, ldb, nullptr, batch, st, 0);
     }
+#endif
+#ifndef BANDLU_TRS_BWD_WINDOW
+    if constexpr (std::is_same_v<AP, Strided<const double>> && KL + KU + 1 <= 32)
+        return launch_trs_bwd_lean<KL, KU>(n, A, ldab, B, batch, st);
 #endif
     return launch_trs_window<KL, KU>(n, 1, A, ldab, P, B, ldb, nullptr, batch, st, 0);
 }
@@ -631,19 +662,21 @@ namespace {
 // e2e call pays no allocation: NS streams and one staging buffer per stream
 // (grown on demand, on the device of the call).
 struct HostPipe {
-    static constexpr int NS = 3;
+    static constexpr int NSMAX = 8;
+    int NS = 4;
     std::mutex mu;
     int dev = -1;
-    cudaStream_t s[NS] = {};
-    cudaEvent_t done[NS] = {};
+    cudaStream_t s[NSMAX] = {};
+    cudaEvent_t done[NSMAX] = {};
     cudaEvent_t start = nullptr;
-    void *buf[NS] = {};
+    void *buf[NSMAX] = {};
     size_t cap = 0;
     cudaError_t prepare(size_t need) {
         int d = 0;
         cudaError_t e = cudaGetDevice(&d);
         if (e != cudaSuccess) return e;
         if (d != dev) {  // first call, or another device: (re)create streams and events
+            if (const char *v = std::getenv("BANDLU_HOST_STREAMS")) NS = std::max(1, std::min(NSMAX, atoi(v)));
             for (int i = 0; i < NS; ++i) buf[i] = nullptr;  // buffers of another device are abandoned
             cap = 0;
             for (int i = 0; i < NS; ++i) {
@@ -693,9 +726,13 @@ extern "C" int dgbsv_strided_batched_host(int n, int kl, int ku, int nrhs, doubl
 
     cudaStream_t user = (cudaStream_t)stream;
     const int64_t bytes_per = strideA * 8 + strideB * 8 + strideP * 4 + 4;
-    // ~64 MB chunks over NS = 3 streams: H2D of chunk c+1, the kernels of chunk c
+    // ~32 MB chunks over NS = 4 streams: H2D of chunk c+1, the kernels of chunk c
     // and D2H of chunk c-1 overlap (PCIe copy engines run both directions at once)
-    int64_t ch = (int64_t)((64ll << 20) / (bytes_per > 0 ? bytes_per : 1));
+    static const long long chunk_mb = [] {
+        const char *v = std::getenv("BANDLU_HOST_CHUNK_MB");
+        return v ? std::max(1ll, atoll(v)) : 32ll;  // measured at C3: 4 x 32 MB 32.0 ms, 3 x 64 MB 33.4 ms
+    }();
+    int64_t ch = (int64_t)((chunk_mb << 20) / (bytes_per > 0 ? bytes_per : 1));
     ch = ch < 1 ? 1 : (ch > batch ? batch : ch);
     const int nchunks = (int)((batch + ch - 1) / ch);
     const size_t offB = (size_t)ch * strideA * 8, offP = offB + (((size_t)ch * strideB * 8 + 15) & ~(size_t)15);
@@ -708,9 +745,9 @@ extern "C" int dgbsv_strided_batched_host(int n, int kl, int ku, int nrhs, doubl
     if ((e = g_pipe.prepare(need)) != cudaSuccess) return cuda_ret(e);
     cudaEvent_t ev0 = g_pipe.start;
     cudaEventRecord(ev0, user);
-    for (int i = 0; i < HostPipe::NS; ++i) cudaStreamWaitEvent(g_pipe.s[i], ev0, 0);
+    for (int i = 0; i < g_pipe.NS; ++i) cudaStreamWaitEvent(g_pipe.s[i], ev0, 0);
     for (int c = 0; c < nchunks; ++c) {
-        const int i = c % HostPipe::NS;
+        const int i = c % g_pipe.NS;
         cudaStream_t si = g_pipe.s[i];
         char *base = (char *)g_pipe.buf[i];
         double *dA = (double *)base, *dB = (double *)(base + offB);
@@ -731,7 +768,7 @@ extern "C" int dgbsv_strided_batched_host(int n, int kl, int ku, int nrhs, doubl
         cudaMemcpyAsync(hinfo + b0, dI, (size_t)cb * 4, cudaMemcpyDeviceToHost, si);
         if ((e = cudaGetLastError()) != cudaSuccess) { ret = cuda_ret(e); break; }
     }
-    for (int i = 0; i < HostPipe::NS; ++i) {
+    for (int i = 0; i < g_pipe.NS; ++i) {
         cudaEventRecord(g_pipe.done[i], g_pipe.s[i]);
         cudaStreamWaitEvent(user, g_pipe.done[i], 0);
     }

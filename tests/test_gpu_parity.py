@@ -154,7 +154,7 @@ def test_trs_parity_sizes(n, kl, ku):
         assert np.all(same_bits(_gpu_trs(A, ipiv, B.copy(), n, kl, ku, variant), Bo))
 
 
-@pytest.mark.parametrize("kl,ku,nrhs", [(2, 2, 1), (10, 10, 1), (2, 32, 16), (5, 6, 3)])
+@pytest.mark.parametrize("kl,ku,nrhs", [(2, 2, 1), (10, 10, 1), (2, 32, 16), (5, 6, 3), (1, 1, 1), (0, 3, 1)])
 def test_gbsv_parity_with_singular(kl, ku, nrhs):
     n, batch = 80, 10
     A = I.gen_band(n, n, kl, ku, count=batch)
