@@ -220,6 +220,50 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
     const unsigned gbits = (G == 32) ? 0xffffffffu : ((1u << G) - 1u);
     const unsigned gbase = (unsigned)(g * G);
     const unsigned below = (1u << t) - 1u;
+#ifdef BANDLU_ROWS_LOOKAHEAD
+    constexpr bool LA = true;
+#else
+    constexpr bool LA = false;
+#endif
+    struct PivState {
+        double x[R];
+        bool cand[R];
+        int pb, rb;
+        unsigned gb;
+    } ps;
+    // IAMAX of step s (column j): first max |x| over the candidate rows, exact
+    // (64-bit key, ties by smallest logical row; reading 2)
+    auto search = [&](int s, int j, PivState &o) {
+        uint64_t kb = 0;
+        int pb = FREE, rb = 0;
+        bool cb = false;
+#pragma unroll
+        for (int ri = 0; ri < R; ++ri) {
+            o.x[ri] = VS(ri, s);
+            o.cand[ri] = (pos[ri] <= j + KL) && (pos[ri] < mloc);
+            const uint64_t k = o.cand[ri] ? abs_key(o.x[ri]) : 0ull;
+            const bool better = o.cand[ri] && (!cb || k > kb || (k == kb && pos[ri] < pb));
+            if (better) {
+                kb = k;
+                pb = pos[ri];
+                rb = ri;
+                cb = true;
+            }
+        }
+        const unsigned hi = (unsigned)(kb >> 32);
+        const unsigned mhi = group_max_u32<G>(hi, g);
+        unsigned gb = (__ballot_sync(0xffffffffu, cb && hi == mhi) >> gbase) & gbits;
+        if (__any_sync(0xffffffffu, live && __popc(gb) != 1)) {
+            // exact tie-break: low word, then smallest logical row (first index)
+            const unsigned lo = (unsigned)kb;
+            const unsigned mlo = group_max_u32<G>((cb && hi == mhi) ? lo : 0u, g);
+            const unsigned pp = group_min_u32<G>((cb && hi == mhi && lo == mlo) ? (unsigned)pb : 0xffffffffu);
+            gb = (__ballot_sync(0xffffffffu, cb && (unsigned)pb == pp) >> gbase) & gbits;
+        }
+        o.pb = pb;
+        o.rb = rb;
+        o.gb = gb;
+    };
 #pragma unroll 1
     for (int j0 = 0; j0 < mn; j0 += U) {
         cp_async_wait<C::DB - 1>();  // rows j0+KL+1 .. j0+KL+U landed (this lane's part)
@@ -249,35 +293,18 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
             const int j = j0 + s;
             if (j >= mn) break;
 
-            // ---- IAMAX over the candidates (logical rows j..min(j+KL, m-1))
+            // ---- IAMAX over the candidates (logical rows j..min(j+KL, m-1)); with LOOKAHEAD
+            // the search of step s > 0 already ran inside step s-1, right after column j's update
+            if (!LA || s == 0) search(s, j, ps);
             double x[R];
             bool cand[R];
-            uint64_t kb = 0;
-            int pb = FREE, rb = 0;
-            bool cb = false;
 #pragma unroll
             for (int ri = 0; ri < R; ++ri) {
-                x[ri] = VS(ri, s);
-                cand[ri] = (pos[ri] <= j + KL) && (pos[ri] < mloc);
-                const uint64_t k = cand[ri] ? abs_key(x[ri]) : 0ull;
-                const bool better = cand[ri] && (!cb || k > kb || (k == kb && pos[ri] < pb));
-                if (better) {
-                    kb = k;
-                    pb = pos[ri];
-                    rb = ri;
-                    cb = true;
-                }
+                x[ri] = ps.x[ri];
+                cand[ri] = ps.cand[ri];
             }
-            const unsigned hi = (unsigned)(kb >> 32);
-            const unsigned mhi = group_max_u32<G>(hi, g);
-            unsigned gb = (__ballot_sync(0xffffffffu, cb && hi == mhi) >> gbase) & gbits;
-            if (__any_sync(0xffffffffu, live && __popc(gb) != 1)) {
-                // exact tie-break: low word, then smallest logical row (first index)
-                const unsigned lo = (unsigned)kb;
-                const unsigned mlo = group_max_u32<G>((cb && hi == mhi) ? lo : 0u, g);
-                const unsigned pp = group_min_u32<G>((cb && hi == mhi && lo == mlo) ? (unsigned)pb : 0xffffffffu);
-                gb = (__ballot_sync(0xffffffffu, cb && (unsigned)pb == pp) >> gbase) & gbits;
-            }
+            const int pb = ps.pb, rb = ps.rb;
+            const unsigned gb = ps.gb;
             const bool is_piv = (t == __ffs(gb) - 1);
 
             // ---- pivot row (U row j: slots s..s+KV) + (B entry, logical row) -> record s
@@ -341,6 +368,11 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
             // 128-bit broadcast reads of slot pairs (2h, 2h+1) covering s+1 .. s+KV: half the
             // load instructions of 64-bit reads for the same shared-memory wavefronts (C3
             // factorization 1.016 -> 0.981 ms)
+            if (LA) {
+#pragma unroll
+                for (int ri = 0; ri < R; ++ri)
+                    if (pslot[ri]) pos[ri] = FREE;
+            }
 #pragma unroll
             for (int h = (s + 1) / 2; h <= (s + KV) / 2; ++h) {
                 const double2 u2 = ld_shared_v2(rcs + h * 16);
@@ -349,6 +381,9 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
                     if (2 * h >= s + 1) VS(ri, 2 * h) = __fma_rn(lu[ri], -u2.x, VS(ri, 2 * h));
                     if (2 * h + 1 <= s + KV) VS(ri, 2 * h + 1) = __fma_rn(lu[ri], -u2.y, VS(ri, 2 * h + 1));
                 }
+                // column j+1 (slot s+1) is final for step j+1: its pivot search overlaps the
+                // rest of this update
+                if (LA && h == (s + 1) / 2 && s + 1 < U && j + 1 < mn) search(s + 1, j + 1, ps);
             }
 #else
 #pragma unroll
