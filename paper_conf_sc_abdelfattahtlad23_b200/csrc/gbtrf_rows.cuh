@@ -62,13 +62,19 @@ struct TrfRows {
     static constexpr int WARPS_FIT = (72 * 1024) / (GPW * GROUP_DBL * 8);
     // wide windows (W > 24) run 8 warps/SM: 2 per scheduler, so each thread may use up to 255
     // registers (the register file is split per scheduler: 3 warps each would cap it at 168)
-    static constexpr int WMAX = W > 24 ? 2 : BANDLU_ROWS_WARPS;
+#ifndef BANDLU_ROWS_WIDE_WARPS
+#define BANDLU_ROWS_WIDE_WARPS 2
+#endif
+#ifndef BANDLU_ROWS_WIDE_MINW
+#define BANDLU_ROWS_WIDE_MINW 8
+#endif
+    static constexpr int WMAX = W > 24 ? BANDLU_ROWS_WIDE_WARPS : BANDLU_ROWS_WARPS;
     static constexpr int WARPS = WARPS_FIT < 1 ? 1 : (WARPS_FIT < WMAX ? WARPS_FIT : WMAX);
 #ifndef BANDLU_ROWS_MINW
 #define BANDLU_ROWS_MINW 12
 #endif
     // resident warps per SM target (wide windows: 8, as the window kernel)
-    static constexpr int MINB = ((W <= 24 ? BANDLU_ROWS_MINW : 8) + WARPS - 1) / WARPS;
+    static constexpr int MINB = ((W <= 24 ? BANDLU_ROWS_MINW : BANDLU_ROWS_WIDE_MINW) + WARPS - 1) / WARPS;
     static constexpr size_t smem_bytes() { return (size_t)WARPS * GPW * GROUP_DBL * sizeof(double); }
 };
 

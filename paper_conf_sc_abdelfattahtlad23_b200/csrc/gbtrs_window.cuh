@@ -70,8 +70,16 @@ struct TrsWin {
 
 // PAIRS: RHS rows staged / stored as 16-byte row pairs (nrhs >= 2); otherwise one
 // 8-byte row per step (nrhs == 1: one lane per matrix, measured faster there).
+#ifndef BANDLU_TRS_MINB
+#define BANDLU_TRS_MINB 1
+#endif
+#ifdef BANDLU_TRS_MAXREG
+#define BANDLU_TRS_BOUNDS __maxnreg__(BANDLU_TRS_MAXREG)
+#else
+#define BANDLU_TRS_BOUNDS __launch_bounds__(32, BANDLU_TRS_MINB)
+#endif
 template <int KL, int KU, bool PAIRS, class AP, class PP, class BP>
-__global__ void __launch_bounds__(32)
+__global__ void BANDLU_TRS_BOUNDS
     gbtrs_window_kernel(int n, int nrhs, AP A, int ldab, PP P, BP B, int ldb, const int *__restrict__ skip_info,
                         int batch, int R /* pow2 lanes per matrix */, int chunks /* rhs chunks per matrix */,
                         int gpw /* matrices (groups) per warp, <= 32 / R */,

@@ -20,7 +20,8 @@ def one(spec):
     name, flags = spec.split("=", 1)
     flags = [f for f in flags.split(",") if f]
     lib = os.path.join(OUT, f"lib_{name}.so")
-    cmd = [_build._nvcc(), *[f for f in _build.NVCC_FLAGS if f != "-v" and f != "-Xptxas"], "-DBANDLU_ONLY_C3",
+    only = [] if name.startswith("F_") else ["-DBANDLU_ONLY_C3"]  # F_*: every band (C4, C5 ...)
+    cmd = [_build._nvcc(), *[f for f in _build.NVCC_FLAGS if f != "-v" and f != "-Xptxas"], *only,
            *flags, _build.SRC, "-o", lib]
     r = subprocess.run(cmd, capture_output=True, text=True)
     return name, r.returncode, r.stderr[-800:]
