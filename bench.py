@@ -385,7 +385,12 @@ def main():
 
     peak, peak_kind = peaks()
     trf_kernel = {bl.ROWS: "gbtrf_rows_kernel", bl.WINDOW: "gbtrf_window_kernel"}.get(v_trf, "gbtrf_generic_kernel")
-    trs_kernel = "gbtrs_window_kernel" if bl.trs_variant(n, kl, ku, nrhs) == bl.WINDOW else "gbtrs_generic_kernel"
+    if fused:  # the backward-only launch of dgbtrfs (bandlu.cu launch_trs_bwd)
+        trs_kernel = ("gbtrs_rows_kernel" if kl + ku + 1 <= 4 else
+                      "gbtrs_bwd_kernel" if kl + ku + 1 <= 32 else "gbtrs_window_kernel")
+    else:
+        trs_kernel = {bl.WINDOW: "gbtrs_window_kernel", bl.ROWS: "gbtrs_rows_kernel"}.get(
+            bl.trs_variant(n, kl, ku, nrhs), "gbtrs_generic_kernel")
     dom = trf_kernel if trf_ms >= trs_ms else trs_kernel
     dom_ms = (trf_ms if trf_ms >= trs_ms else trs_ms) / args.steps
     dom_bytes = cnt * (k_trf if trf_ms >= trs_ms else k_trs)
