@@ -41,7 +41,7 @@
 #endif
 
 #ifndef BANDLU_TRS_NS_WIDE
-#define BANDLU_TRS_NS_WIDE 8
+#define BANDLU_TRS_NS_WIDE 4
 #endif
 
 namespace bandlu {
@@ -70,13 +70,14 @@ struct TrsWin {
 
 // PAIRS: RHS rows staged / stored as 16-byte row pairs (nrhs >= 2); otherwise one
 // 8-byte row per step (nrhs == 1: one lane per matrix, measured faster there).
-#ifndef BANDLU_TRS_MINB
-#define BANDLU_TRS_MINB 1
-#endif
-#ifdef BANDLU_TRS_MAXREG
+// experiments: BANDLU_TRS_MAXREG (register cap) or BANDLU_TRS_MINB (resident CTAs); the default
+// bound lets ptxas pick (C4: 128 registers; (32, 1) picked more and ran 2.83 vs 2.16 ms)
+#if defined(BANDLU_TRS_MAXREG)
 #define BANDLU_TRS_BOUNDS __maxnreg__(BANDLU_TRS_MAXREG)
-#else
+#elif defined(BANDLU_TRS_MINB)
 #define BANDLU_TRS_BOUNDS __launch_bounds__(32, BANDLU_TRS_MINB)
+#else
+#define BANDLU_TRS_BOUNDS __launch_bounds__(32)
 #endif
 template <int KL, int KU, bool PAIRS, class AP, class PP, class BP>
 __global__ void BANDLU_TRS_BOUNDS
