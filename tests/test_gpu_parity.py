@@ -319,6 +319,29 @@ def test_trfs_fused_matches_trf_then_trs(kl, ku, nrhs):
     assert np.all(np.isnan(Bg.cpu().numpy()[:, :, n:]))  # ldb padding untouched
 
 
+@pytest.mark.parametrize("kl,ku", [(0, 0), (1, 1), (2, 3), (4, 4), (10, 10), (2, 32), (32, 32)])
+@pytest.mark.parametrize("n", [1, 2, 5, 20, 21, 22, 33, 64])
+def test_trfs_fused_small_n_ragged_batch(kl, ku, n):
+    """dgbtrfs at n below / around the window length (the backward solve reads
+    rows < 0 from pad slots for its last kv steps) and a batch that leaves the
+    last warp partly empty, bitwise vs oracle dgbtrf + dgbtrs."""
+    batch = 13
+    A = I.gen_band(n, n, kl, ku, count=batch)
+    B = I.gen_rhs(n, 1, ldb=n + 3, count=batch)
+    Ao, Bo = A.copy(), B.copy()
+    ipo, info_o = oracle.dgbtrf(Ao, n, n, kl, ku)
+    oracle.dgbtrs(Ao, ipo, Bo, n, kl, ku)
+    Ag = torch.from_numpy(A).cuda(); Bg = torch.from_numpy(B).cuda()
+    P = torch.zeros((batch, n), dtype=torch.int32, device="cuda")
+    inf = torch.zeros(batch, dtype=torch.int32, device="cuda")
+    bl.dgbtrfs_strided_batched(n, kl, ku, Ag, P, Bg, inf)
+    torch.cuda.synchronize()
+    assert np.array_equal(inf.cpu().numpy(), info_o)
+    assert np.array_equal(P.cpu().numpy(), ipo)
+    assert np.all(same_bits(Ag.cpu().numpy(), Ao))
+    assert np.all(same_bits(Bg.cpu().numpy(), Bo))  # incl. the NaN padding rows of ldb
+
+
 @pytest.mark.parametrize("kl,ku,nrhs", [(2, 3, 2), (10, 10, 1), (1, 1, 3), (0, 4, 1), (4, 0, 2), (2, 32, 16), (33, 20, 1)])
 @pytest.mark.parametrize("trans", ["T", "C"])
 def test_trs_transposed_parity(kl, ku, nrhs, trans):
