@@ -88,7 +88,10 @@ enum bandlu_variant {
                            where compiled.  dgbtrs ('N'): one lane per RHS row, a group of
                            pow2 >= kl+ku+1 lanes per (matrix, RHS column), compiled (kl, ku) with
                            kl+ku+1 <= 32 only (bandlu_trs_rows_available); AUTO's choice for
-                           nrhs == 1 with kl+ku+1 <= 4.  Bitwise equal results */
+                           nrhs == 1 with kl+ku+1 <= 4.  Bitwise equal results */,
+    BANDLU_THREAD = 5   /* dgbtrf only: one thread per matrix, the whole (kl+1) x (kl+ku+1) window in
+                           registers, thin compiled bands (bandlu_thread_available); bitwise equal
+                           results */
 };
 
 /* ---- dgbtrf: band LU with partial pivoting ---- */
@@ -187,6 +190,8 @@ int bandlu_trs_variant(int n, int kl, int ku, int nrhs);
 int bandlu_tc_available(int kl, int ku);
 /* 1 if a row-slot (BANDLU_ROWS) factorization kernel is compiled for (kl, ku), else 0. */
 int bandlu_rows_available(int kl, int ku);
+/* 1 if a thread-per-matrix factorization kernel (BANDLU_THREAD) is compiled for (kl, ku), else 0. */
+int bandlu_thread_available(int kl, int ku);
 /* 1 if a lane-per-row solve kernel (dgbtrs BANDLU_ROWS) is compiled for (kl, ku), else 0. */
 int bandlu_trs_rows_available(int kl, int ku);
 /* ABI version of this library. */

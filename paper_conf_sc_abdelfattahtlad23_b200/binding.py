@@ -18,7 +18,7 @@ import torch
 
 from . import _build
 
-AUTO, GENERIC, WINDOW, TC, ROWS = 0, 1, 2, 3, 4
+AUTO, GENERIC, WINDOW, TC, ROWS, THREAD = 0, 1, 2, 3, 4, 5
 ERR_UNSUPPORTED, ERR_CUDA = 1000, 2000
 
 _lib = None
@@ -70,6 +70,7 @@ def load(build_if_missing: bool = False):
         "bandlu_tc_available": [i, i],
         "bandlu_rows_available": [i, i],
         "bandlu_trs_rows_available": [i, i],
+        "bandlu_thread_available": [i, i],
         "bandlu_trs_variant": [i, i, i, i],
         "bandlu_version": [],
     }
@@ -84,7 +85,7 @@ def load(build_if_missing: bool = False):
 # exported symbol list (checked by tests against include/bandlu.h)
 EXPORTS = ("dgbtrf_batched", "dgbtrf_strided_batched", "dgbtrf_strided_batched_ex", "dgbtrs_batched",
            "dgbtrs_strided_batched", "dgbtrs_strided_batched_ex", "dgbsv_batched", "dgbsv_strided_batched",
-           "dgbsv_strided_batched_host", "dgbtrfs_strided_batched", "dgbtrfs_strided_batched_ex", "bandlu_trf_variant", "bandlu_trs_variant", "bandlu_tc_available", "bandlu_rows_available", "bandlu_trs_rows_available",
+           "dgbsv_strided_batched_host", "dgbtrfs_strided_batched", "dgbtrfs_strided_batched_ex", "bandlu_trf_variant", "bandlu_trs_variant", "bandlu_tc_available", "bandlu_rows_available", "bandlu_trs_rows_available", "bandlu_thread_available",
            "bandlu_version")
 
 
@@ -213,6 +214,11 @@ def tc_available(kl: int, ku: int) -> bool:
 def rows_available(kl: int, ku: int) -> bool:
     """True if a row-slot factorization kernel (variant ROWS) is compiled for (kl, ku)."""
     return bool(load().bandlu_rows_available(kl, ku))
+
+
+def thread_available(kl: int, ku: int) -> bool:
+    """True if a thread-per-matrix factorization kernel (variant THREAD) is compiled for (kl, ku)."""
+    return bool(load().bandlu_thread_available(kl, ku))
 
 
 def trs_rows_available(kl: int, ku: int) -> bool:

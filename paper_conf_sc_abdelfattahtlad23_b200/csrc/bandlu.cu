@@ -17,6 +17,7 @@
 #include "gbtrf_rows.cuh"
 #include "gbtrf_wide.cuh"
 #include "gbtrf_tc.cuh"
+#include "gbtrf_thread.cuh"
 #include "gbtrf_window.cuh"
 #include "gbtrs_bwd.cuh"
 #include "gbtrs_rows.cuh"
@@ -78,6 +79,27 @@ namespace {
     X(10, 10, BANDLU_ROWS_C3_G, BANDLU_ROWS_C3_R)        \
     X(10, 7, 16, 1)                                      \
     X(2, 32, 8, 1)
+#endif
+
+// (KL, KU) compiled as thread-per-matrix factorization kernels (gbtrf_thread.cuh, thin
+// bands); BANDLU_THREAD_AUTO_LIST: the ones AUTO prefers (measured)
+#ifdef BANDLU_ONLY_C3
+#define BANDLU_THREAD_LIST(X) X(1, 1)
+#else
+#define BANDLU_THREAD_LIST(X) \
+    X(0, 0)                   \
+    X(0, 3)                   \
+    X(1, 1)                   \
+    X(2, 2)                   \
+    X(2, 3)                   \
+    X(3, 0)                   \
+    X(3, 2)                   \
+    X(4, 4)
+#endif
+#if defined(BANDLU_THREAD_AUTO_ALL)  // experiments: every compiled thin band
+#define BANDLU_THREAD_AUTO_LIST(X) BANDLU_THREAD_LIST(X)
+#elif !defined(BANDLU_THREAD_AUTO_LIST)
+#define BANDLU_THREAD_AUTO_LIST(X)
 #endif
 
 // (KL, KU) with kl+1 > 32: two-warp row-slot kernel (gbtrf_wide.cuh), dispatched as
@@ -162,6 +184,16 @@ int launch_trf_wide(int m, int n, AP A, int ldab, PP P, int *info, int batch, cu
     return cuda_ret(cudaGetLastError());
 }
 
+template <int KL, int KU, bool FWD, class AP, class PP, class BP>
+int launch_trf_thread(int m, int n, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st, BP B) {
+    using C = TrfThread<KL, KU>;
+    const unsigned grid = (unsigned)((batch + C::THREADS - 1) / C::THREADS);
+    auto k = gbtrf_thread_kernel<KL, KU, FWD, AP, PP, BP>;
+    if (int r = set_smem(k, C::smem_bytes())) return r;
+    k<<<grid, C::THREADS, C::smem_bytes(), st>>>(m, n, A, ldab, P, info, batch, B);
+    return cuda_ret(cudaGetLastError());
+}
+
 template <class AP, class PP>
 int launch_trf_generic(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st) {
     const unsigned grid = (unsigned)(((int64_t)batch * 32 + 127) / 128);
@@ -209,6 +241,21 @@ bool trs_rows_available(int kl, int ku) {
     return false;
 }
 
+bool trf_thread_available(int kl, int ku) {
+#define X(a, b) \
+    if (kl == a && ku == b) return true;
+    BANDLU_THREAD_LIST(X)
+#undef X
+    return false;
+}
+bool trf_thread_preferred(int kl, int ku) {
+#define X(a, b) \
+    if (kl == a && ku == b) return true;
+    BANDLU_THREAD_AUTO_LIST(X)
+#undef X
+    return false;
+}
+
 bool trf_tc_available(int kl, int ku) {
 #define X(a, b) \
     if (kl == a && ku == b) return true;
@@ -221,6 +268,7 @@ int pick_trf(int m, int n, int kl, int ku) {
     if (m <= 0 || n <= 0) return BANDLU_GENERIC;
     // BANDLU_TC is opt-in: measured slower than the row-owner window at C3
     // (1.54 vs 1.10 ms), so AUTO never picks it.
+    if (trf_thread_preferred(kl, ku)) return BANDLU_THREAD;
     if (trf_rows_available(kl, ku)) return BANDLU_ROWS;
     return trf_window_available(kl, ku) ? BANDLU_WINDOW : BANDLU_GENERIC;
 }
@@ -247,6 +295,13 @@ int run_trf(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int b
 #undef X
         return BANDLU_ERR_UNSUPPORTED;
     }
+    if (variant == BANDLU_THREAD && m > 0 && n > 0) {
+#define X(a, b) \
+    if (kl == a && ku == b) return launch_trf_thread<a, b, false>(m, n, A, ldab, P, info, batch, st, Strided<double>{nullptr, 0});
+        BANDLU_THREAD_LIST(X)
+#undef X
+        return BANDLU_ERR_UNSUPPORTED;
+    }
     if (variant == BANDLU_ROWS && m > 0 && n > 0) {
 #define X(a, b, g, r) \
     if (kl == a && ku == b) return launch_trf_rows<a, b, g, r, false>(m, n, A, ldab, P, info, batch, st, Strided<double>{nullptr, 0});
@@ -265,7 +320,8 @@ int run_trf(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int b
 #undef X
         return BANDLU_ERR_UNSUPPORTED;
     }
-    if (variant != BANDLU_GENERIC && variant != BANDLU_WINDOW && variant != BANDLU_TC && variant != BANDLU_ROWS)
+    if (variant != BANDLU_GENERIC && variant != BANDLU_WINDOW && variant != BANDLU_TC && variant != BANDLU_ROWS &&
+        variant != BANDLU_THREAD)
         return BANDLU_ERR_UNSUPPORTED;
     return launch_trf_generic(m, n, kl, ku, A, ldab, P, info, batch, st);
 }
@@ -413,6 +469,17 @@ int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ld
         int r = BANDLU_ERR_UNSUPPORTED;
         Strided<const double> Ac{A.base, A.stride};
         Strided<const int> Pc{P.base, P.stride};
+        if (trf_thread_preferred(kl, ku)) {
+#define X(a, b)                                                                                           \
+    if (kl == a && ku == b) {                                                                             \
+        r = 0;                                                                                            \
+        if (phase != 2) r = launch_trf_thread<a, b, true>(n, n, A, ldab, P, info, batch, st, B);          \
+        if (r == 0 && phase != 1) r = launch_trs_bwd<a, b>(n, Ac, ldab, Pc, B, ldb, batch, st);           \
+    }
+            BANDLU_THREAD_LIST(X)
+#undef X
+            return r;
+        }
         if (trf_rows_available(kl, ku)) {
 #define X(a, b, g, rr)                                                                                    \
     if (kl == a && ku == b) {                                                                             \
@@ -518,6 +585,7 @@ int bandlu_version(void) { return 1; }
 int bandlu_trf_variant(int m, int n, int kl, int ku) { return pick_trf(m, n, kl, ku); }
 int bandlu_tc_available(int kl, int ku) { return trf_tc_available(kl, ku) ? 1 : 0; }
 int bandlu_rows_available(int kl, int ku) { return trf_rows_available(kl, ku) ? 1 : 0; }
+int bandlu_thread_available(int kl, int ku) { return trf_thread_available(kl, ku) ? 1 : 0; }
 int bandlu_trs_rows_available(int kl, int ku) { return trs_rows_available(kl, ku) ? 1 : 0; }
 int bandlu_trs_variant(int n, int kl, int ku, int nrhs) { return pick_trs(n, kl, ku, nrhs); }
 

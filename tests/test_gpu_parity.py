@@ -45,6 +45,8 @@ def trf_variants(kl, ku):
         v.append(bl.ROWS)
     if bl.tc_available(kl, ku):
         v.append(bl.TC)
+    if bl.thread_available(kl, ku):
+        v.append(bl.THREAD)
     return v
 
 
@@ -61,7 +63,7 @@ def _check_trf(m, n, kl, ku, batch, variant, ldab=None, first=0, A_in=None):
 
 
 @pytest.mark.parametrize("kl,ku", ALL_BANDS)
-@pytest.mark.parametrize("variant", [bl.WINDOW, bl.GENERIC, bl.ROWS, bl.TC])
+@pytest.mark.parametrize("variant", [bl.WINDOW, bl.GENERIC, bl.ROWS, bl.TC, bl.THREAD])
 @pytest.mark.parametrize("n", [1, 2, 7, 37, 100])
 def test_trf_parity_small(kl, ku, variant, n):
     if variant not in trf_variants(kl, ku):
