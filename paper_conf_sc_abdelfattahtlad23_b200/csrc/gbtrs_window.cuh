@@ -36,6 +36,8 @@
 #pragma once
 #include "common.cuh"
 
+#include <type_traits>
+
 #ifndef BANDLU_TRS_NS_NARROW
 #define BANDLU_TRS_NS_NARROW 16
 #endif
@@ -291,13 +293,32 @@ __global__ void BANDLU_TRS_BOUNDS
             cp_async_wait<NS - 1>();
             __syncwarp();
             const double *uc = fac_ptr(k) - max(0, KV - j);  // uc[r] = AB(r, j), r >= KV - j valid
+            // U column as 16-byte pairs when its smem parity is the same on every lane (strided
+            // batches with an even stride): half the load instructions
+            const uint32_t ua = smem_u32(uc);
+            const bool pe = __all_sync(0xffffffffu, ((ua >> 3) & 1u) == 0u);
+            const bool po = !pe && __all_sync(0xffffffffu, ((ua >> 3) & 1u) == 1u);
             double xj = x[s];
             if (xj != 0.0) {
                 xj = __ddiv_rn(xj, uc[KV]);
                 // rows j-i < 0 (last KV steps) read the pad / neighbouring slot: they only
                 // feed window slots of rows < 0, which are never stored (dead slots)
+                auto pairs = [&](auto par) {  // element e = KV - i; pair (e0, e0+1) 16-byte aligned
 #pragma unroll
-                for (int i = 1; i < WB; ++i) x[s + i] = __fma_rn(-xj, uc[KV - i], x[s + i]);
+                    for (int e0 = -decltype(par)::value; e0 < KV; e0 += 2) {
+                        const double2 u2 = ld_shared_v2(ua + (uint32_t)(e0 * 8));
+                        if (e0 >= 0) x[s + KV - e0] = __fma_rn(-xj, u2.x, x[s + KV - e0]);
+                        if (e0 + 1 < KV) x[s + KV - e0 - 1] = __fma_rn(-xj, u2.y, x[s + KV - e0 - 1]);
+                    }
+                };
+                if (pe) {
+                    pairs(std::integral_constant<int, 0>{});
+                } else if (po) {
+                    pairs(std::integral_constant<int, 1>{});
+                } else {
+#pragma unroll
+                    for (int i = 1; i < WB; ++i) x[s + i] = __fma_rn(-xj, uc[KV - i], x[s + i]);
+                }
             }
             // result x_j: rows (j, j+1) leave as one 16-byte store
             if (!PAIRS) {
