@@ -75,10 +75,18 @@ namespace {
 #elif defined(BANDLU_ONLY_C3)
 #define BANDLU_ROWS_LIST(X) X(10, 10, BANDLU_ROWS_C3_G, BANDLU_ROWS_C3_R)
 #else
+// thin bands as row-slot kernels too (G*R >= kl+1+4 with the window kernel's G): measured
+// C2 (1,1) 0.156 -> 0.149 ms, C1 (2,2) 0.028 -> 0.026 ms, XGC-like (4,4) 0.077 -> 0.058 ms
+#ifdef BANDLU_NO_ROWS_THIN
+#define BANDLU_ROWS_THIN_LIST(X)
+#else
+#define BANDLU_ROWS_THIN_LIST(X) X(1, 1, 8, 1) X(2, 2, 8, 1) X(2, 3, 8, 1) X(4, 4, 16, 1)
+#endif
 #define BANDLU_ROWS_LIST(X)                              \
     X(10, 10, BANDLU_ROWS_C3_G, BANDLU_ROWS_C3_R)        \
     X(10, 7, 16, 1)                                      \
-    X(2, 32, 8, 1)
+    X(2, 32, 8, 1)                                       \
+    BANDLU_ROWS_THIN_LIST(X)
 #endif
 
 // (KL, KU) compiled as thread-per-matrix factorization kernels (gbtrf_thread.cuh, thin

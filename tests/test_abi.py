@@ -109,9 +109,11 @@ def test_gbsv_argument_errors(lib):
 def test_variant_heuristic_is_shape_only(lib):
     from paper_conf_sc_abdelfattahtlad23_b200 import binding as b
     assert b.trf_variant(512, 512, 10, 10) == b.ROWS
-    assert b.rows_available(10, 10) and b.rows_available(2, 32) and not b.rows_available(1, 1)
+    assert b.rows_available(10, 10) and b.rows_available(2, 32) and b.rows_available(1, 1)
+    assert not b.rows_available(0, 3) and not b.rows_available(3, 0)
     assert b.tc_available(10, 10) and not b.tc_available(1, 1)  # opt-in tensor-core kernel
-    assert b.trf_variant(256, 256, 1, 1) == b.WINDOW
+    assert b.trf_variant(256, 256, 1, 1) == b.ROWS  # thin bands: row-slot kernel too
+    assert b.trf_variant(64, 64, 0, 3) == b.WINDOW
     assert b.trf_variant(100, 100, 32, 32) == b.ROWS  # kl+1 > 32 lanes: two-warp row-slot kernel
     assert b.trf_variant(100, 100, 33, 20) == b.GENERIC  # band not compiled: safeguard kernel
     assert b.trs_variant(100, 32, 32, 1) == b.WINDOW
