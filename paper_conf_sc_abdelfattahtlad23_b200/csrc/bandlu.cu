@@ -379,7 +379,11 @@ int launch_trs_generic(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP
 // (the window solve one per 32/R matrices); it only wins where a warp packs
 // >= 8 matrices (kl+ku+1 <= 4): measured C2 (1,1) 0.097 vs 0.105 ms, but C3
 // (10,10) 0.78 vs 0.32 ms and PELE-like (10,10) 0.083 vs 0.039 ms.
+#ifdef BANDLU_NO_TRS_ROWS_AUTO  // experiments
+bool trs_rows_preferred(int, int) { return false; }
+#else
 bool trs_rows_preferred(int kl, int ku) { return kl + ku + 1 <= 4 && trs_rows_available(kl, ku); }
+#endif
 
 int pick_trs(int n, int kl, int ku, int nrhs) {
     (void)n;
