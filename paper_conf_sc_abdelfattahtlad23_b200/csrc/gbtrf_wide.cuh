@@ -191,11 +191,21 @@ __global__ void __launch_bounds__(64, 4)
                 if (is_piv) bv[j] = y;
                 if (y != 0.0) bq = __fma_rn(lu, -y, bq);
             }
+#ifndef BANDLU_WIDE_LDS64
+            // 128-bit broadcast reads of slot pairs (as gbtrf_rows.cuh): half the load instructions
+#pragma unroll
+            for (int h = (s + 1) / 2; h <= (s + KV) / 2; ++h) {
+                const double2 u2 = ld_shared_v2(rcs + h * 16);
+                if (2 * h >= s + 1) VS(2 * h) = __fma_rn(lu, -u2.x, VS(2 * h));
+                if (2 * h + 1 <= s + KV) VS(2 * h + 1) = __fma_rn(lu, -u2.y, VS(2 * h + 1));
+            }
+#else
 #pragma unroll
             for (int k = 1; k <= KV; ++k) {
                 const double uk = ld_volatile_shared_f64(rcs + (s + k) * 8);
                 VS(s + k) = __fma_rn(lu, -uk, VS(s + k));
             }
+#endif
             if (is_piv) pos = FREE;
             colj += ldab;
             ++ipj;
