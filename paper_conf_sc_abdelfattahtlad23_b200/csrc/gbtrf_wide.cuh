@@ -23,7 +23,10 @@ template <int KL_, int KU_>
 struct TrfWide {
     static constexpr int KL = KL_, KU = KU_, KV = KL + KU, W = KV + 1;
     static constexpr int G = 64;                 // lanes per matrix (= the CTA)
-    static constexpr int U = 4;
+#ifndef BANDLU_WIDE_U
+#define BANDLU_WIDE_U 4
+#endif
+    static constexpr int U = BANDLU_WIDE_U;
     static constexpr int WS = W + U, H = (WS + 1) / 2;
     static_assert(KL + 1 + U <= G, "slots");
     static constexpr int WPB = 2 * H + 4;
