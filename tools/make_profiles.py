@@ -112,11 +112,12 @@ def main():
         summary[c] = s
         md.append(f"## {c}")
         md.append("")
-        md.append("| kernel | us | DRAM read GB | DRAM write GB | DRAM % | issue % | FP64 pipe % | regs | top stalls |")
+        md.append("| kernel | us | DRAM read GB | DRAM write GB | DRAM GB/s | issue % | FP64 pipe % | regs | top stalls |")
         md.append("|---|---|---|---|---|---|---|---|---|")
         for k, d in s.items():
             md.append(f"| {k} | {d.get('duration_us', 0):.1f} | {d.get('dram_bytes_read', 0)/1e9:.3f} | "
-                      f"{d.get('dram_bytes_write', 0)/1e9:.3f} | {d.get('dram_throughput_pct', 0):.1f} | "
+                      f"{d.get('dram_bytes_write', 0)/1e9:.3f} | "
+                      f"{(d.get('dram_bytes_read', 0) + d.get('dram_bytes_write', 0)) / max(d.get('duration_us', 1), 1e-9) / 1e3:.0f} | "
                       f"{d.get('issue_active_pct', 0):.1f} | {d.get('fp64_pipe_pct', 0):.1f} | {d.get('registers', 0):.0f} | "
                       + ", ".join(f"{h} {p}%" for h, p in d["top_stalls_pct"].items()) + " |")
         md.append("")
