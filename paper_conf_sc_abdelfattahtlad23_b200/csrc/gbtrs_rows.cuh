@@ -28,7 +28,9 @@
 //    is two shuffles; rows that retire are stored, and at the end of the
 //    forward pass the lanes hold rows n-G..n-1, which is exactly the backward
 //    pass's starting window -- no reload.
-// 32/G (matrix, RHS column) units per warp; no shared memory, ~40 registers: 64 warps per SM.
+// 32/G (matrix, RHS column) units per warp; no shared memory, 64-72 registers.  Measured:
+// AUTO for kl+ku+1 <= 4 only: it issues one division per matrix-step,
+// the window solve one per warp-step for up to 32 matrices.
 #pragma once
 #include "common.cuh"
 
