@@ -223,6 +223,13 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
     double *colj = live ? ab + KV : nullptr;  // &AB(KV, j)
     double *colb = live ? ab : nullptr;       // &AB(0, j0)
     int *ipj = ipiv;
+    int pv[U];     // the block's pivots (1-based), stored once per block by lane 0 of the group
+    double yv[U];  // FWD: the block's y(j), likewise
+#pragma unroll
+    for (int s = 0; s < U; ++s) {
+        pv[s] = 0;
+        yv[s] = 0.0;
+    }
     const unsigned gbits = (G == 32) ? 0xffffffffu : ((1u << G) - 1u);
     const unsigned gbase = (unsigned)(g * G);
     const unsigned below = (1u << t) - 1u;
@@ -341,7 +348,11 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
             const double p = ld_volatile_shared_f64(rcs + s * 8);
 #endif
             const bool zp = (p == 0.0);
+#ifndef BANDLU_ROWS_IPIV_STEP
+            pv[s] = ppos + 1;  // stored once per block (C3 factorization 0.979 -> 0.960 ms)
+#else
             if (is_piv) *ipj = ppos + 1;
+#endif
             if (live && zp && linfo == 0) linfo = j + 1;
 
             // ---- interchange = relabel; the pivot slot retires after this step
@@ -363,7 +374,11 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
             }
             if constexpr (FWD) {
                 const double y = yp.x;
+#ifdef BANDLU_ROWS_Y_BLOCK
+                yv[s] = y;
+#else
                 if (is_piv) bv[j] = y;
+#endif
                 if (y != 0.0) {
 #pragma unroll
                     for (int ri = 0; ri < R; ++ri) bq[ri] = __fma_rn(lu[ri], -y, bq[ri]);
@@ -426,6 +441,33 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
             }
         }
         colb += (int64_t)U * ldab;
+#ifndef BANDLU_ROWS_IPIV_STEP
+        if (live && t == 0) {
+            int *ip = ipiv + j0;
+            if (U == 4 && j0 + U <= mn && (reinterpret_cast<uintptr_t>(ip) & 15) == 0) {
+                *reinterpret_cast<int4 *>(ip) = make_int4(pv[0], pv[1 % U], pv[2 % U], pv[3 % U]);
+            } else {
+#pragma unroll
+                for (int s = 0; s < U; ++s)
+                    if (j0 + s < mn) ip[s] = pv[s];
+            }
+        }
+#endif
+#ifdef BANDLU_ROWS_Y_BLOCK
+        if constexpr (FWD) {
+            if (live && t == 0) {
+                double *yp4 = bv + j0;
+                if (U == 4 && j0 + U <= mn && (reinterpret_cast<uintptr_t>(yp4) & 15) == 0) {
+                    reinterpret_cast<double2 *>(yp4)[0] = make_double2(yv[0], yv[1 % U]);
+                    reinterpret_cast<double2 *>(yp4)[1] = make_double2(yv[2 % U], yv[3 % U]);
+                } else {
+#pragma unroll
+                    for (int s = 0; s < U; ++s)
+                        if (j0 + s < mn) yp4[s] = yv[s];
+                }
+            }
+        }
+#endif
         __syncwarp();
         // shift the window by U columns: slot r <- slot r+U
 #pragma unroll
