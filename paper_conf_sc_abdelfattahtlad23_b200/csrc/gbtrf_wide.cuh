@@ -122,7 +122,9 @@ __global__ void __launch_bounds__(64, 4)
     const int mn = min(m, n);
     double *colj = ab + KV;
     double *colb = ab;
-    int *ipj = ipiv;
+    int pv[U];  // the block's pivots (1-based), stored once per block by thread 0 (as gbtrf_rows.cuh)
+#pragma unroll
+    for (int s = 0; s < U; ++s) pv[s] = 0;
     const unsigned below = (1u << lane) - 1u;
 #pragma unroll 1
     for (int j0 = 0; j0 < mn; j0 += U) {
@@ -181,7 +183,7 @@ __global__ void __launch_bounds__(64, 4)
             const int ppos = (int)__double_as_longlong(yp.y);
             const double p = ld_volatile_shared_f64(rcs + s * 8);
             const bool zp = (p == 0.0);
-            if (is_piv) *ipj = ppos + 1;
+            pv[s] = ppos + 1;
             if (zp && linfo == 0) linfo = j + 1;
             if (pos == j && !is_piv) pos = ppos;  // interchange = relabel
 
@@ -211,7 +213,6 @@ __global__ void __launch_bounds__(64, 4)
 #endif
             if (is_piv) pos = FREE;
             colj += ldab;
-            ++ipj;
         }
         // ---- U rows j0 .. j0+U-1 -> HBM (32-byte column chunks)
         __syncthreads();
@@ -222,6 +223,16 @@ __global__ void __launch_bounds__(64, 4)
                 colb[boff(k) + KV] = ld_shared_f64(rec_s + (uint32_t)((bs * WP + bk) * 8));
         }
         colb += (int64_t)U * ldab;
+        if (t == 0) {
+            int *ip = ipiv + j0;
+            if (U == 4 && j0 + U <= mn && (reinterpret_cast<uintptr_t>(ip) & 15) == 0) {
+                *reinterpret_cast<int4 *>(ip) = make_int4(pv[0], pv[1 % U], pv[2 % U], pv[3 % U]);
+            } else {
+#pragma unroll
+                for (int s = 0; s < U; ++s)
+                    if (j0 + s < mn) ip[s] = pv[s];
+            }
+        }
         __syncthreads();
 #pragma unroll
         for (int h = 0; h < H; ++h) {
