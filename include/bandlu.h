@@ -50,12 +50,18 @@
  *
  * ------------------------------------------------------------- errors
  * Return 0: work enqueued.  Return -k: argument k (1-based position in the
- * C signature) is illegal; LAPACK numbering is kept where LAPACK has the
- * argument (trf: -1 m, -2 n, -3 kl, -4 ku, -6 ldab; trs: -1 trans, -2 n,
- * -3 kl, -4 ku, -5 nrhs, -7 ldab, -10 ldb; gbsv: -1 n, -2 kl, -3 ku,
- * -4 nrhs, -6 ldab, -9 ldb); batch < 0, a NULL array with batch > 0, or a
- * too-small stride return the position of that argument.  Nothing is
- * enqueued when the return is nonzero.  BANDLU_ERR_UNSUPPORTED: a forced
+ * C signature) is illegal; batch < 0, a NULL array with batch > 0, or a
+ * too-small stride return the position of that argument too.  For the
+ * pointer-array variants the positions are LAPACK's numbering (trf: -1 m,
+ * -2 n, -3 kl, -4 ku, -6 ldab; trs: -1 trans, -2 n, -3 kl, -4 ku, -5 nrhs,
+ * -7 ldab, -10 ldb; gbsv: -1 n, -2 kl, -3 ku, -4 nrhs, -6 ldab, -9 ldb).
+ * The strided variants insert stride arguments, so later positions shift:
+ * dgbtrf_strided -5 dA, -6 ldab, -7 strideA, -8 dipiv, -9 strideP, -10 dinfo,
+ * -11 batch; dgbtrs_strided -7 ldab, -8 strideA, -9 dipiv, -10 strideP,
+ * -11 dB, -12 ldb, -13 strideB, -14 batch; dgbsv_strided / dgbtrfs_strided /
+ * dgbsv_strided_host -5 dA, -6 ldab, -7 strideA, -8 dipiv, -9 strideP,
+ * -10 dB, -11 ldb, -12 strideB, -13 dinfo, -14 batch.  Nothing is enqueued
+ * when the return is nonzero.  BANDLU_ERR_UNSUPPORTED: a forced
  * variant that is not compiled for the shape.  BANDLU_ERR_CUDA +
  * (cudaError_t) : a launch/runtime error (enqueue failed).
  */
@@ -121,7 +127,11 @@ int dgbtrs_strided_batched(char trans, int n, int kl, int ku, int nrhs,
                            int batch, bandlu_stream_t stream);
 
 /* ---- dgbsv: dgbtrf + dgbtrs.  B is untouched for every matrix
- * with info > 0 (LAPACK DGBSV). ---- */
+ * with info > 0 (LAPACK DGBSV).  Strided, nrhs == 1, a band with a row-slot
+ * kernel and y(0..n-1) fitting in shared memory: ONE launch of the fused gbsv
+ * kernel (factorization, forward substitution on the fly, backward
+ * substitution by the same lanes; Sec. 7 P:686-702 generalised to any n).
+ * Otherwise a factorization launch and a solve launch. ---- */
 int dgbsv_batched(int n, int kl, int ku, int nrhs,
                   double *const *dA_array, int ldab, int *const *dipiv_array,
                   double *const *dB_array, int ldb, int *dinfo,
@@ -134,19 +144,23 @@ int dgbsv_strided_batched(int n, int kl, int ku, int nrhs,
 
 /* ---- dgbtrfs: dgbtrf followed by dgbtrs('N') on every matrix, as one call
  * (the bench's hot-path step).  Same arguments and numbering as
- * dgbsv_strided_batched.  For nrhs == 1 and a compiled (kl, ku) the forward
- * substitution is fused into the factorization kernel (the paper's fused
- * GBSV on the augmented [A|B], Sec. 7), followed by one
- * backward-substitution launch; results are bitwise those of the separate
- * calls.  Unlike dgbsv, B is solved also where info > 0 (as dgbtrs would:
- * singular U gives Inf/NaN). ---- */
+ * dgbsv_strided_batched.  nrhs == 1 and a band with a row-slot kernel: ONE
+ * launch (the fused kernel, as dgbsv; y in shared memory when it fits, else
+ * in B).  nrhs == 1 and another compiled (kl, ku): the factorization kernel
+ * applies the forward substitution (the paper's augmented [A|B], Sec. 7
+ * P:688-702), then one backward-substitution launch.  Results are bitwise
+ * those of the separate calls.  Unlike dgbsv, B is solved also where
+ * info > 0 (as dgbtrs would: singular U gives Inf/NaN). ---- */
 int dgbtrfs_strided_batched(int n, int kl, int ku, int nrhs,
                             double *dA, int ldab, int64_t strideA,
                             int *dipiv, int64_t strideP,
                             double *dB, int ldb, int64_t strideB, int *dinfo,
                             int batch, bandlu_stream_t stream);
-/* phase (profiling): 0 = everything, 1 = factorization (+ fused forward
- * solve) only, 2 = the remaining solve only; any other value returns -16. */
+/* phase (profiling): 0 = everything, 1 = the first launch only, 2 = the second
+ * launch only (nothing when the plan has one launch); + BANDLU_TRFS_TWO_LAUNCH
+ * forces the two-launch plan (factorization + forward, then backward); any
+ * other value returns -16. */
+#define BANDLU_TRFS_TWO_LAUNCH 16
 int dgbtrfs_strided_batched_ex(int n, int kl, int ku, int nrhs,
                                double *dA, int ldab, int64_t strideA,
                                int *dipiv, int64_t strideP,
@@ -154,9 +168,10 @@ int dgbtrfs_strided_batched_ex(int n, int kl, int ku, int nrhs,
                                int batch, bandlu_stream_t stream, int phase);
 
 /* ---- host-buffer end-to-end variant of dgbsv_strided_batched: hA, hipiv,
- * hB, hinfo are HOST pointers (pinned memory recommended).  The library keeps
- * three streams and three ~64 MB device staging buffers per process (created
- * on first use on the current device, grown on demand, never freed), copies
+ * hB, hinfo are HOST pointers (pinned memory recommended).  The library keeps,
+ * per device, four streams and four staging buffers of one ~32 MB batch chunk
+ * each (created on first use on that device, grown on demand, never freed;
+ * BANDLU_HOST_STREAMS / BANDLU_HOST_CHUNK_MB override the defaults), copies
  * A and B in, factors and solves, copies A (factors), ipiv, B (solution) and
  * info back, and synchronizes `stream` before returning.  Batch chunks are
  * pipelined so host->device copies, kernels and device->host copies overlap.
@@ -186,14 +201,24 @@ int bandlu_trf_variant(int m, int n, int kl, int ku);
 int bandlu_trs_variant(int n, int kl, int ku, int nrhs);
 /* 1 if a tensor-core (BANDLU_TC) factorization kernel is compiled for (kl, ku),
  * else 0 (no launch).  BANDLU_TC is never chosen by AUTO; force it with
- * dgbtrf_strided_batched_ex. */
+ * dgbtrf_strided_batched_ex.  Compiled only in -DBANDLU_WITH_TC builds. */
 int bandlu_tc_available(int kl, int ku);
 /* 1 if a row-slot (BANDLU_ROWS) factorization kernel is compiled for (kl, ku), else 0. */
 int bandlu_rows_available(int kl, int ku);
-/* 1 if a thread-per-matrix factorization kernel (BANDLU_THREAD) is compiled for (kl, ku), else 0. */
+/* 1 if a thread-per-matrix factorization kernel (BANDLU_THREAD) is compiled for (kl, ku), else 0
+ * (only in -DBANDLU_WITH_THREAD builds: measured slower, AUTO never picks it). */
 int bandlu_thread_available(int kl, int ku);
 /* 1 if a lane-per-row solve kernel (dgbtrs BANDLU_ROWS) is compiled for (kl, ku), else 0. */
 int bandlu_trs_rows_available(int kl, int ku);
+/* The launches one dgbtrfs_strided_batched call makes for a shape (no launch):
+ * returns their number L (0..2; < 0 on a negative argument) and, if kinds is
+ * not NULL, writes L codes kinds[i] = 16 * kernel + bytes, kernel: 1 gbtrf_rows,
+ * 2 gbtrf_window, 3 gbtrf_wide, 4 gbtrf_thread, 5 gbtrf_generic, 6 gbtrs_bwd,
+ * 7 gbtrs_rows, 8 gbtrs_window, 9 gbtrs_generic; bytes (what the launch must
+ * move per matrix): 1 factorization, 2 factorization + forward
+ * substitution, 3 backward substitution, 4 full solve, 5 fused gbsv.
+ * two_launch != 0: the plan of phase | BANDLU_TRFS_TWO_LAUNCH. */
+int bandlu_trfs_plan(int n, int kl, int ku, int nrhs, int two_launch, int *kinds);
 /* ABI version of this library. */
 int bandlu_version(void);
 

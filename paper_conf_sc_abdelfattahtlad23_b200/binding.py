@@ -72,6 +72,7 @@ def load(build_if_missing: bool = False):
         "bandlu_trs_rows_available": [i, i],
         "bandlu_thread_available": [i, i],
         "bandlu_trs_variant": [i, i, i, i],
+        "bandlu_trfs_plan": [i, i, i, i, i, p],
         "bandlu_version": [],
     }
     for name, args in sig.items():
@@ -86,7 +87,7 @@ def load(build_if_missing: bool = False):
 EXPORTS = ("dgbtrf_batched", "dgbtrf_strided_batched", "dgbtrf_strided_batched_ex", "dgbtrs_batched",
            "dgbtrs_strided_batched", "dgbtrs_strided_batched_ex", "dgbsv_batched", "dgbsv_strided_batched",
            "dgbsv_strided_batched_host", "dgbtrfs_strided_batched", "dgbtrfs_strided_batched_ex", "bandlu_trf_variant", "bandlu_trs_variant", "bandlu_tc_available", "bandlu_rows_available", "bandlu_trs_rows_available", "bandlu_thread_available",
-           "bandlu_version")
+           "bandlu_trfs_plan", "bandlu_version")
 
 
 def _stream(stream):
@@ -111,13 +112,31 @@ def _dev(t: torch.Tensor, dtype, name: str, ndim: int):
         raise TypeError(f"{name}: need a contiguous CUDA {dtype} tensor of rank {ndim}")
 
 
+def _shapes(A: torch.Tensor, n: int, ipiv: torch.Tensor | None, npiv: int, B: torch.Tensor | None = None,
+            info: torch.Tensor | None = None) -> None:
+    """Every tensor must describe the same batch on the same device: A [batch, n, ldab],
+    ipiv [batch, >= npiv], B [batch, nrhs, ldb], info [batch] (the library trusts the
+    sizes it is given, so a mismatch here would be an out-of-bounds access there)."""
+    batch = A.shape[0]
+    if A.shape[1] != n:
+        raise ValueError(f"A.shape[1] = {A.shape[1]} must be n = {n}")
+    for t, nm in ((ipiv, "ipiv"), (B, "B"), (info, "info")):
+        if t is None:
+            continue
+        if t.shape[0] != batch:
+            raise ValueError(f"{nm}.shape[0] = {t.shape[0]} must equal the batch {batch}")
+        if t.device != A.device:
+            raise ValueError(f"{nm} is on {t.device}, A on {A.device}")
+    if ipiv is not None and ipiv.shape[1] < max(1, npiv):
+        raise ValueError(f"ipiv.shape[1] = {ipiv.shape[1]} < {max(1, npiv)}")
+
+
 def dgbtrf_strided_batched(m: int, n: int, kl: int, ku: int, A: torch.Tensor, ipiv: torch.Tensor,
                            info: torch.Tensor, variant: int = AUTO, stream=None) -> None:
     """In place: A [batch, n, ldab] -> LU factors; ipiv [batch, >=min(m,n)]; info [batch]."""
     _dev(A, torch.float64, "A", 3); _dev(ipiv, torch.int32, "ipiv", 2); _dev(info, torch.int32, "info", 1)
     batch, n_, ldab = A.shape
-    if n_ != n:
-        raise ValueError("A.shape[1] must be n")
+    _shapes(A, n, ipiv, min(m, n), info=info)
     f = load().dgbtrf_strided_batched_ex
     _chk("dgbtrf_strided_batched", f(m, n, kl, ku, _ptr(A), ldab, n * ldab, _ptr(ipiv), ipiv.shape[1],
                                      _ptr(info), batch, _stream(stream), variant))
@@ -127,6 +146,7 @@ def dgbtrs_strided_batched(trans: str, n: int, kl: int, ku: int, A: torch.Tensor
                            B: torch.Tensor, variant: int = AUTO, stream=None) -> None:
     """In place: B [batch, nrhs, ldb] <- A^{-1} B using dgbtrf factors."""
     _dev(A, torch.float64, "A", 3); _dev(ipiv, torch.int32, "ipiv", 2); _dev(B, torch.float64, "B", 3)
+    _shapes(A, n, ipiv, n, B=B)
     batch, _, ldab = A.shape
     _, nrhs, ldb = B.shape
     f = load().dgbtrs_strided_batched_ex
@@ -138,6 +158,7 @@ def dgbsv_strided_batched(n: int, kl: int, ku: int, A: torch.Tensor, ipiv: torch
                           info: torch.Tensor, stream=None) -> None:
     _dev(A, torch.float64, "A", 3); _dev(ipiv, torch.int32, "ipiv", 2); _dev(B, torch.float64, "B", 3)
     _dev(info, torch.int32, "info", 1)
+    _shapes(A, n, ipiv, n, B=B, info=info)
     batch, _, ldab = A.shape
     _, nrhs, ldb = B.shape
     _chk("dgbsv_strided_batched", load().dgbsv_strided_batched(
@@ -151,6 +172,7 @@ def dgbtrfs_strided_batched(n: int, kl: int, ku: int, A: torch.Tensor, ipiv: tor
     phase 1 / 2 run only the factorization / only the solve launch (profiling)."""
     _dev(A, torch.float64, "A", 3); _dev(ipiv, torch.int32, "ipiv", 2); _dev(B, torch.float64, "B", 3)
     _dev(info, torch.int32, "info", 1)
+    _shapes(A, n, ipiv, n, B=B, info=info)
     batch, _, ldab = A.shape
     _, nrhs, ldb = B.shape
     _chk("dgbtrfs_strided_batched", load().dgbtrfs_strided_batched_ex(
@@ -190,6 +212,7 @@ def dgbsv_strided_batched_host(n: int, kl: int, ku: int, A: torch.Tensor, ipiv: 
                      (info, torch.int32, "info")):
         if t.is_cuda or t.dtype != d or not t.is_contiguous():
             raise TypeError(f"{nm}: need a contiguous host {d} tensor")
+    _shapes(A, n, ipiv, n, B=B, info=info)
     batch, _, ldab = A.shape
     _, nrhs, ldb = B.shape
     _chk("dgbsv_strided_batched_host", load().dgbsv_strided_batched_host(
@@ -228,3 +251,21 @@ def trs_rows_available(kl: int, ku: int) -> bool:
 
 def trs_variant(n: int, kl: int, ku: int, nrhs: int) -> int:
     return load().bandlu_trs_variant(n, kl, ku, nrhs)
+
+
+KERNEL_NAMES = {1: "gbtrf_rows_kernel", 2: "gbtrf_window_kernel", 3: "gbtrf_wide_kernel", 4: "gbtrf_thread_kernel",
+                5: "gbtrf_generic_kernel", 6: "gbtrs_bwd_kernel", 7: "gbtrs_rows_kernel", 8: "gbtrs_window_kernel",
+                9: "gbtrs_generic_kernel"}
+BYTE_KINDS = {1: "trf", 2: "trf_fwd", 3: "trs_bwd", 4: "trs", 5: "gbsv"}
+TRFS_TWO_LAUNCH = 16
+
+
+def trfs_plan(n: int, kl: int, ku: int, nrhs: int, two_launch: bool = False) -> dict:
+    """The launches one dgbtrfs_strided_batched call makes for a shape (bandlu_trfs_plan)."""
+    kinds = (ctypes.c_int * 4)()
+    k = load().bandlu_trfs_plan(n, kl, ku, nrhs, int(two_launch), kinds)
+    if k < 0:
+        raise BandLUError("bandlu_trfs_plan", k)
+    codes = list(kinds)[:k]
+    return {"kernels": [KERNEL_NAMES[c >> 4] for c in codes], "bytes": [BYTE_KINDS[c & 15] for c in codes],
+            "fused": k == 1 and (codes[0] & 15) == 5}

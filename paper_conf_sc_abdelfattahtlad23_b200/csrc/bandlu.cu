@@ -51,10 +51,11 @@ namespace {
     X(2, 32)
 // (KL, KU) pairs also compiled as tensor-core (DMMA) factorization kernels
 // (kl+1 <= 16; preferred by AUTO where compiled).
-#ifdef BANDLU_NO_TC
-#define BANDLU_TC_LIST(X)
-#else
+// opt-in experiment (-DBANDLU_WITH_TC): measured slower than the row-slot kernel, AUTO never picks it
+#ifdef BANDLU_WITH_TC
 #define BANDLU_TC_LIST(X) X(10, 10)
+#else
+#define BANDLU_TC_LIST(X)
 #endif
 #endif
 
@@ -91,7 +92,11 @@ namespace {
 
 // (KL, KU) compiled as thread-per-matrix factorization kernels (gbtrf_thread.cuh, thin
 // bands); BANDLU_THREAD_AUTO_LIST: the ones AUTO prefers (measured)
-#ifdef BANDLU_ONLY_C3
+// opt-in experiment (-DBANDLU_WITH_THREAD): measured slower than the row-slot kernels for every
+// thin band, AUTO never picks it
+#if !defined(BANDLU_WITH_THREAD)
+#define BANDLU_THREAD_LIST(X)
+#elif defined(BANDLU_ONLY_C3)
 #define BANDLU_THREAD_LIST(X) X(1, 1)
 #else
 #define BANDLU_THREAD_LIST(X) \
@@ -170,11 +175,11 @@ int launch_trf_window(int m, int n, AP A, int ldab, PP P, int *info, int batch, 
     return cuda_ret(cudaGetLastError());
 }
 
-template <int KL, int KU, int G, int R, bool FWD, class AP, class PP, class BP>
+template <int KL, int KU, int G, int R, int FL, class AP, class PP, class BP>
 int launch_trf_rows(int m, int n, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st, BP B) {
     using C = TrfRows<KL, KU, G, R>;
-    auto k = gbtrf_rows_kernel<KL, KU, G, R, FWD, AP, PP, BP>;
-    size_t sm = C::smem_bytes();
+    auto k = gbtrf_rows_kernel<KL, KU, G, R, FL, AP, PP, BP>;
+    size_t sm = (FL & FL_YSM) ? C::smem_bytes_y(n) : C::smem_bytes();
     if (int r = set_smem(k, sm)) return r;
     const int64_t per_block = (int64_t)C::WARPS * C::GPW;
     const unsigned grid = (unsigned)((batch + per_block - 1) / per_block);
@@ -312,7 +317,7 @@ int run_trf(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int b
     }
     if (variant == BANDLU_ROWS && m > 0 && n > 0) {
 #define X(a, b, g, r) \
-    if (kl == a && ku == b) return launch_trf_rows<a, b, g, r, false>(m, n, A, ldab, P, info, batch, st, Strided<double>{nullptr, 0});
+    if (kl == a && ku == b) return launch_trf_rows<a, b, g, r, 0>(m, n, A, ldab, P, info, batch, st, Strided<double>{nullptr, 0});
         BANDLU_ROWS_LIST(X)
 #undef X
 #define X(a, b) \
@@ -466,17 +471,91 @@ int launch_trs_bwd(int n, AP A, int ldab, PP P, BP B, int ldb, int batch, cudaSt
 }
 
 // ------------------------------------- fused factor + solve (dgbtrf; dgbtrs)
-// nrhs == 1 with a compiled window: ONE factorization launch that also applies
-// the forward substitution (FWD), then the backward-only solve launch.
-// Otherwise the plain trf + trs pair.  Results equal dgbtrf followed by
-// dgbtrs('N') for every matrix (B is solved even where info > 0).
-// phase: 0 = both launches, 1 = factorization (+ fused forward solve) only,
-// 2 = solve only (backward, or the full solve when not fused) -- 1/2 let the
-// bench time the two kernels separately with events between them.
+// nrhs == 1 on a band with a row-slot kernel: ONE launch (the fused gbsv
+// kernel: factorization, forward substitution on the fly, backward
+// substitution by the same lanes, Sec. 7).
+// y(0..n-1) sits in shared memory when it fits next to the row ring at the
+// kernel's resident-CTA target, else in B.  Other compiled bands with
+// nrhs == 1: the factorization kernel with the forward substitution, then the
+// backward-only solve launch.  Otherwise the plain trf + trs pair.
+// Results equal dgbtrf followed by dgbtrs('N') for every matrix (dgbtrfs
+// solves B even where info > 0; dgbsv leaves B untouched there).
+// phase: 0 = every launch, 1 = first launch only, 2 = second launch only (the
+// bench times them separately); | TRFS_TWO_LAUNCH forces the two-launch plan.
+constexpr int TRFS_TWO_LAUNCH = BANDLU_TRFS_TWO_LAUNCH;
+constexpr size_t kSmemPerSM = 227 * 1024;
+
+template <int KL, int KU, int G, int R>
+bool rows_ysm_fits(int n) {
+    using C = TrfRows<KL, KU, G, R>;
+    const size_t b = C::smem_bytes_y(n);
+    return b <= kSmemPerSM && b * (size_t)C::MINB <= kSmemPerSM;
+}
+
+bool rows_fused_available(int kl, int ku) {
+#define X(a, b, g, r) \
+    if (kl == a && ku == b) return true;
+    BANDLU_ROWS_LIST(X)
+#undef X
+    return false;
+}
+
+bool rows_ysm_fits_rt(int n, int kl, int ku) {
+#define X(a, b, g, r) \
+    if (kl == a && ku == b) return rows_ysm_fits<a, b, g, r>(n);
+    BANDLU_ROWS_LIST(X)
+#undef X
+    return false;
+}
+
+// kernel ids / byte classes reported by bandlu_trfs_plan (include/bandlu.h)
+enum { KN_TRF_ROWS = 1, KN_TRF_WINDOW, KN_TRF_WIDE, KN_TRF_THREAD, KN_TRF_GENERIC, KN_TRS_BWD, KN_TRS_ROWS,
+       KN_TRS_WINDOW, KN_TRS_GENERIC };
+enum { KB_TRF = 1, KB_TRF_FWD, KB_TRS_BWD, KB_TRS, KB_GBSV };
+
+// the launches one dgbtrfs call makes for the shape (what run_trfs does)
+int trfs_plan(int n, int kl, int ku, int nrhs, bool two_launch, int *kinds) {
+    int k = 0;
+    auto put = [&](int name, int bytes) { if (kinds) kinds[k] = name * 16 + bytes; ++k; };
+    if (n <= 0 || nrhs <= 0) return 0;
+    if (nrhs == 1 && !two_launch && rows_fused_available(kl, ku)) {
+        put(KN_TRF_ROWS, KB_GBSV);
+        return k;
+    }
+    if (nrhs == 1 && (trf_window_available(kl, ku) || trf_wide_available(kl, ku))) {
+        const int tv = trf_thread_preferred(kl, ku) ? KN_TRF_THREAD
+                       : trf_wide_available(kl, ku) ? KN_TRF_WIDE
+                       : trf_rows_available(kl, ku) ? KN_TRF_ROWS : KN_TRF_WINDOW;
+        put(tv, KB_TRF_FWD);
+        put(kl + ku + 1 <= 4 && trs_rows_preferred(kl, ku) ? KN_TRS_ROWS
+            : kl + ku + 1 <= 32 ? KN_TRS_BWD : KN_TRS_WINDOW, KB_TRS_BWD);
+        return k;
+    }
+    const int tv = pick_trf(n, n, kl, ku);
+    put(tv == BANDLU_ROWS ? (trf_wide_available(kl, ku) ? KN_TRF_WIDE : KN_TRF_ROWS)
+        : tv == BANDLU_WINDOW ? KN_TRF_WINDOW : tv == BANDLU_THREAD ? KN_TRF_THREAD : KN_TRF_GENERIC, KB_TRF);
+    const int sv = pick_trs(n, kl, ku, nrhs);
+    put(sv == BANDLU_ROWS ? KN_TRS_ROWS : sv == BANDLU_WINDOW ? KN_TRS_WINDOW : KN_TRS_GENERIC, KB_TRS);
+    return k;
+}
+
 template <class AP, class PP, class BP>
 int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ldb, int *info, int batch,
              cudaStream_t st, int phase) {
+    const bool two = (phase & TRFS_TWO_LAUNCH) != 0;
+    phase &= ~TRFS_TWO_LAUNCH;
     if (batch == 0) return 0;
+    if (n > 0 && nrhs == 1 && !two && rows_fused_available(kl, ku)) {
+        if (phase == 2) return 0;  // the whole path is the first (only) launch
+        const bool ysm = rows_ysm_fits_rt(n, kl, ku);
+#define X(a, b, g, rr)                                                                                               \
+    if (kl == a && ku == b)                                                                                          \
+        return ysm ? launch_trf_rows<a, b, g, rr, FL_FWD | FL_BWD | FL_YSM>(n, n, A, ldab, P, info, batch, st, B) \
+                   : launch_trf_rows<a, b, g, rr, FL_FWD | FL_BWD>(n, n, A, ldab, P, info, batch, st, B);
+        BANDLU_ROWS_LIST(X)
+#undef X
+        return BANDLU_ERR_UNSUPPORTED;
+    }
     if (n > 0 && nrhs == 1 && (trf_window_available(kl, ku) || trf_wide_available(kl, ku))) {
         int r = BANDLU_ERR_UNSUPPORTED;
         Strided<const double> Ac{A.base, A.stride};
@@ -496,8 +575,8 @@ int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ld
 #define X(a, b, g, rr)                                                                                    \
     if (kl == a && ku == b) {                                                                             \
         r = 0;                                                                                            \
-        if (phase != 2) r = launch_trf_rows<a, b, g, rr, true>(n, n, A, ldab, P, info, batch, st, B);     \
-        if (r == 0 && phase != 1) r = launch_trs_bwd<a, b>(n, Ac, ldab, Pc, B, ldb, batch, st); \
+        if (phase != 2) r = launch_trf_rows<a, b, g, rr, FL_FWD>(n, n, A, ldab, P, info, batch, st, B);   \
+        if (r == 0 && phase != 1) r = launch_trs_bwd<a, b>(n, Ac, ldab, Pc, B, ldb, batch, st);           \
     }
             BANDLU_ROWS_LIST(X)
 #undef X
@@ -505,7 +584,7 @@ int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ld
     if (kl == a && ku == b) {                                                                             \
         r = 0;                                                                                            \
         if (phase != 2) r = launch_trf_wide<a, b, true>(n, n, A, ldab, P, info, batch, st, B);           \
-        if (r == 0 && phase != 1) r = launch_trs_bwd<a, b>(n, Ac, ldab, Pc, B, ldb, batch, st); \
+        if (r == 0 && phase != 1) r = launch_trs_bwd<a, b>(n, Ac, ldab, Pc, B, ldb, batch, st);           \
     }
             BANDLU_WIDE_LIST(X)
 #undef X
@@ -515,7 +594,7 @@ int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ld
     if (kl == a && ku == b) {                                                                             \
         r = 0;                                                                                            \
         if (phase != 2) r = launch_trf_window<a, b, true>(n, n, A, ldab, P, info, batch, st, B);          \
-        if (r == 0 && phase != 1) r = launch_trs_bwd<a, b>(n, Ac, ldab, Pc, B, ldb, batch, st); \
+        if (r == 0 && phase != 1) r = launch_trs_bwd<a, b>(n, Ac, ldab, Pc, B, ldb, batch, st);           \
     }
         BANDLU_WINDOW_LIST(X)
 #undef X
@@ -526,6 +605,25 @@ int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ld
     if (phase == 1) return 0;
     return run_trs(n, kl, ku, nrhs, Strided<const double>{A.base, A.stride}, ldab, Strided<const int>{P.base, P.stride},
                    B, ldb, nullptr, batch, st, BANDLU_AUTO);
+}
+
+// dgbsv (strided): the fused single-launch kernel writes B only where info == 0
+// (FL_SKIPI, y in shared memory); otherwise trf, then trs skipping info > 0.
+template <class AP, class PP, class BP>
+int run_gbsv(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ldb, int *info, int batch,
+             cudaStream_t st) {
+    if (batch == 0) return 0;
+    if (n > 0 && nrhs == 1 && rows_fused_available(kl, ku) && rows_ysm_fits_rt(n, kl, ku)) {
+#define X(a, b, g, rr)                                                                                  \
+    if (kl == a && ku == b)                                                                             \
+        return launch_trf_rows<a, b, g, rr, FL_FWD | FL_BWD | FL_YSM | FL_SKIPI>(n, n, A, ldab, P, info, \
+                                                                                 batch, st, B);
+        BANDLU_ROWS_LIST(X)
+#undef X
+    }
+    if (int r = run_trf(n, n, kl, ku, A, ldab, P, info, batch, st, BANDLU_AUTO)) return r;
+    return run_trs(n, kl, ku, nrhs, Strided<const double>{A.base, A.stride}, ldab,
+                   Strided<const int>{P.base, P.stride}, B, ldb, info, batch, st, BANDLU_AUTO);
 }
 
 // ------------------------------------------------------------ arg checks
@@ -600,6 +698,10 @@ int bandlu_rows_available(int kl, int ku) { return trf_rows_available(kl, ku) ? 
 int bandlu_thread_available(int kl, int ku) { return trf_thread_available(kl, ku) ? 1 : 0; }
 int bandlu_trs_rows_available(int kl, int ku) { return trs_rows_available(kl, ku) ? 1 : 0; }
 int bandlu_trs_variant(int n, int kl, int ku, int nrhs) { return pick_trs(n, kl, ku, nrhs); }
+int bandlu_trfs_plan(int n, int kl, int ku, int nrhs, int two_launch, int *kinds) {
+    if (n < 0 || kl < 0 || ku < 0 || nrhs < 0) return -1;
+    return trfs_plan(n, kl, ku, nrhs, two_launch != 0, kinds);
+}
 
 int dgbtrf_strided_batched_ex(int m, int n, int kl, int ku, double *dA, int ldab, int64_t strideA, int *dipiv,
                               int64_t strideP, int *dinfo, int batch, bandlu_stream_t stream, int variant) {
@@ -666,12 +768,8 @@ int dgbsv_strided_batched(int n, int kl, int ku, int nrhs, double *dA, int ldab,
         if (strideB < (int64_t)ldb * nrhs) return -12;
         if (!dinfo) return -13;
     }
-    cudaStream_t st = (cudaStream_t)stream;
-    if (int r = run_trf(n, n, kl, ku, Strided<double>{dA, strideA}, ldab, Strided<int>{dipiv, strideP}, dinfo, batch,
-                        st, BANDLU_AUTO))
-        return r;
-    return run_trs(n, kl, ku, nrhs, Strided<const double>{dA, strideA}, ldab, Strided<const int>{dipiv, strideP},
-                   Strided<double>{dB, strideB}, ldb, dinfo, batch, st, BANDLU_AUTO);
+    return run_gbsv(n, kl, ku, nrhs, Strided<double>{dA, strideA}, ldab, Strided<int>{dipiv, strideP},
+                    Strided<double>{dB, strideB}, ldb, dinfo, batch, (cudaStream_t)stream);
 }
 
 int dgbtrfs_strided_batched_ex(int n, int kl, int ku, int nrhs, double *dA, int ldab, int64_t strideA, int *dipiv,
@@ -694,7 +792,7 @@ int dgbtrfs_strided_batched_ex(int n, int kl, int ku, int nrhs, double *dA, int 
         if (strideB < (int64_t)ldb * nrhs) return -12;
         if (!dinfo) return -13;
     }
-    if (phase < 0 || phase > 2) return -16;
+    if ((phase & ~TRFS_TWO_LAUNCH) < 0 || (phase & ~TRFS_TWO_LAUNCH) > 2) return -16;
     return run_trfs(n, kl, ku, nrhs, Strided<double>{dA, strideA}, ldab, Strided<int>{dipiv, strideP},
                     Strided<double>{dB, strideB}, ldb, dinfo, batch, (cudaStream_t)stream, phase);
 }
@@ -734,37 +832,34 @@ int dgbsv_batched(int n, int kl, int ku, int nrhs, double *const *dA_array, int 
 }  // extern "C"
 
 // ============================================= host-buffer end-to-end path
-// Pipelined over batch chunks on two internal streams: H2D(A_c, B_c) ->
-// gbtrf -> gbtrs -> D2H(A_c, ipiv_c, B_c, info_c); chunk c+1's copies overlap
-// chunk c's kernels (separate copy engines for each direction).
+// Pipelined over batch chunks on NS internal streams: H2D(A_c, B_c) ->
+// dgbsv (one fused launch where available) -> D2H(A_c, ipiv_c, B_c, info_c);
+// chunk c+1's copies overlap chunk c's kernels (separate copy engines for each
+// direction).
 namespace {
 // Device-side state of the host-buffer entry point, kept across calls so an
-// e2e call pays no allocation: NS streams and one staging buffer per stream
-// (grown on demand, on the device of the call).
-struct HostPipe {
+// e2e call pays no allocation: per device, NS streams and one staging buffer
+// per stream (grown on demand).  A process that alternates devices keeps one
+// set per device instead of abandoning the previous one.
+struct DevPipe {
     static constexpr int NSMAX = 8;
-    int NS = 4;
-    std::mutex mu;
-    int dev = -1;
+    int NS = 0;  // 0 = not created yet
     cudaStream_t s[NSMAX] = {};
     cudaEvent_t done[NSMAX] = {};
     cudaEvent_t start = nullptr;
     void *buf[NSMAX] = {};
     size_t cap = 0;
     cudaError_t prepare(size_t need) {
-        int d = 0;
-        cudaError_t e = cudaGetDevice(&d);
-        if (e != cudaSuccess) return e;
-        if (d != dev) {  // first call, or another device: (re)create streams and events
-            if (const char *v = std::getenv("BANDLU_HOST_STREAMS")) NS = std::max(1, std::min(NSMAX, atoi(v)));
-            for (int i = 0; i < NS; ++i) buf[i] = nullptr;  // buffers of another device are abandoned
-            cap = 0;
-            for (int i = 0; i < NS; ++i) {
+        cudaError_t e;
+        if (NS == 0) {
+            int ns = 4;
+            if (const char *v = std::getenv("BANDLU_HOST_STREAMS")) ns = std::max(1, std::min(NSMAX, atoi(v)));
+            for (int i = 0; i < ns; ++i) {
                 if ((e = cudaStreamCreateWithFlags(&s[i], cudaStreamNonBlocking)) != cudaSuccess) return e;
                 if ((e = cudaEventCreateWithFlags(&done[i], cudaEventDisableTiming)) != cudaSuccess) return e;
             }
             if ((e = cudaEventCreateWithFlags(&start, cudaEventDisableTiming)) != cudaSuccess) return e;
-            dev = d;
+            NS = ns;
         }
         if (need > cap) {
             for (int i = 0; i < NS; ++i) {
@@ -781,6 +876,11 @@ struct HostPipe {
         }
         return cudaSuccess;
     }
+};
+struct HostPipe {
+    static constexpr int MAXDEV = 64;
+    std::mutex mu;
+    DevPipe dev[MAXDEV];
 };
 HostPipe g_pipe;
 }  // namespace
@@ -820,16 +920,19 @@ extern "C" int dgbsv_strided_batched_host(int n, int kl, int ku, int nrhs, doubl
     const size_t need = offI + (size_t)ch * 4 + 16;
 
     std::lock_guard<std::mutex> lock(g_pipe.mu);
-    int ret = 0;
+    int ret = 0, d = 0;
     cudaError_t e;
-    if ((e = g_pipe.prepare(need)) != cudaSuccess) return cuda_ret(e);
-    cudaEvent_t ev0 = g_pipe.start;
+    if ((e = cudaGetDevice(&d)) != cudaSuccess) return cuda_ret(e);
+    if (d < 0 || d >= HostPipe::MAXDEV) return BANDLU_ERR_UNSUPPORTED;
+    DevPipe &pp = g_pipe.dev[d];
+    if ((e = pp.prepare(need)) != cudaSuccess) return cuda_ret(e);
+    cudaEvent_t ev0 = pp.start;
     cudaEventRecord(ev0, user);
-    for (int i = 0; i < g_pipe.NS; ++i) cudaStreamWaitEvent(g_pipe.s[i], ev0, 0);
+    for (int i = 0; i < pp.NS; ++i) cudaStreamWaitEvent(pp.s[i], ev0, 0);
     for (int c = 0; c < nchunks; ++c) {
-        const int i = c % g_pipe.NS;
-        cudaStream_t si = g_pipe.s[i];
-        char *base = (char *)g_pipe.buf[i];
+        const int i = c % pp.NS;
+        cudaStream_t si = pp.s[i];
+        char *base = (char *)pp.buf[i];
         double *dA = (double *)base, *dB = (double *)(base + offB);
         int *dP = (int *)(base + offP), *dI = (int *)(base + offI);
         const int64_t b0 = (int64_t)c * ch;
@@ -848,9 +951,9 @@ extern "C" int dgbsv_strided_batched_host(int n, int kl, int ku, int nrhs, doubl
         cudaMemcpyAsync(hinfo + b0, dI, (size_t)cb * 4, cudaMemcpyDeviceToHost, si);
         if ((e = cudaGetLastError()) != cudaSuccess) { ret = cuda_ret(e); break; }
     }
-    for (int i = 0; i < g_pipe.NS; ++i) {
-        cudaEventRecord(g_pipe.done[i], g_pipe.s[i]);
-        cudaStreamWaitEvent(user, g_pipe.done[i], 0);
+    for (int i = 0; i < pp.NS; ++i) {
+        cudaEventRecord(pp.done[i], pp.s[i]);
+        cudaStreamWaitEvent(user, pp.done[i], 0);
     }
     if ((e = cudaStreamSynchronize(user)) != cudaSuccess && !ret) ret = cuda_ret(e);
     return ret;

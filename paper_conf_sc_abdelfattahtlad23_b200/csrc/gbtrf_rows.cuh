@@ -27,6 +27,7 @@
 // Interchanges are relabelings (reading 10), IAMAX is first-max
 // (exact 64-bit key compare, ties by smallest logical row; reading 2).
 #pragma once
+#include "backsolve_fused.cuh"
 #include "common.cuh"
 
 #ifndef BANDLU_ROWS_WARPS
@@ -76,7 +77,18 @@ struct TrfRows {
     // resident warps per SM target (wide windows: 8, as the window kernel)
     static constexpr int MINB = ((W <= 24 ? BANDLU_ROWS_MINW : BANDLU_ROWS_WIDE_MINW) + WARPS - 1) / WARPS;
     static constexpr size_t smem_bytes() { return (size_t)WARPS * GPW * GROUP_DBL * sizeof(double); }
+    // fused solve with y in shared memory: each group also holds y(0..n-1)
+    __host__ __device__ static constexpr int ypad(int n) { return (n + 15) & ~15; }
+    static constexpr size_t smem_bytes_y(int n) { return (size_t)WARPS * GPW * (GROUP_DBL + ypad(n)) * sizeof(double); }
 };
+
+// Kernel modes (template FL, bit flags):
+//   FL_FWD: forward substitution of one right-hand side on the fly (y = L^-1 P b);
+//   FL_BWD: then the backward substitution in the same kernel (backsolve_fused.cuh):
+//           one launch computes dgbtrf + dgbtrs('N') = the fused gbsv kernel;
+//   FL_YSM: y kept in shared memory (n doubles per matrix) instead of B;
+//   FL_SKIPI: B written only where info == 0 (dgbsv; needs FL_YSM).
+enum : int { FL_FWD = 1, FL_BWD = 2, FL_YSM = 4, FL_SKIPI = 8 };
 
 // max of a 32-bit value over the G lanes of each group (all 32 lanes call)
 template <int G>
@@ -106,10 +118,14 @@ __device__ __forceinline__ unsigned group_min_u32(unsigned v) {
 #else
 #define BANDLU_ROWS_BOUNDS(...) __launch_bounds__(__VA_ARGS__::WARPS * 32, __VA_ARGS__::MINB)
 #endif
-template <int KL, int KU, int G, int R, bool FWD, class AP, class PP, class BP>
+template <int KL, int KU, int G, int R, int FL, class AP, class PP, class BP>
 __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
     gbtrf_rows_kernel(int m, int n, AP A, int ldab, PP P, int *__restrict__ info, int batch, BP Bv) {
     using C = TrfRows<KL, KU, G, R>;
+    constexpr bool FWD = FL & FL_FWD, BWD = FL & FL_BWD, YSM = FL & FL_YSM, SKIPI = FL & FL_SKIPI;
+    static_assert(!BWD || FWD, "the fused backward solve needs the forward pass");
+    static_assert(!YSM || BWD, "y in shared memory only with the fused backward solve");
+    static_assert(!SKIPI || YSM, "dgbsv semantics (B untouched where info > 0) need y off B");
     constexpr int KV = C::KV, U = C::U, H = C::H, WP = C::WP, RP = C::RP, D = C::D, RR = C::RR, BK = C::BK,
                   BIT = C::BIT;
     constexpr int FREE = 0x7fffffff;
@@ -129,7 +145,9 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
         return;
     }
     const int mloc = live ? m : 0;
-    double *ring = smem + (size_t)(wib * C::GPW + g) * C::GROUP_DBL;
+    const int gpitch = C::GROUP_DBL + (YSM ? C::ypad(n) : 0);
+    double *ring = smem + (size_t)(wib * C::GPW + g) * gpitch;
+    const uint32_t ybuf_s = smem_u32(ring) + C::GROUP_DBL * 8;  // YSM: y(0..n-1)
     const uint32_t ring_s = smem_u32(ring);
     const uint32_t rec_s = ring_s + RR * WP * 8;
     const double *safe = live ? ab : g_dummy;
@@ -377,7 +395,8 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
 #ifdef BANDLU_ROWS_Y_BLOCK
                 yv[s] = y;
 #else
-                if (is_piv) bv[j] = y;
+                if constexpr (YSM) st_shared_f64_if(is_piv, ybuf_s + (uint32_t)j * 8u, y);
+                else if (is_piv) bv[j] = y;
 #endif
                 if (y != 0.0) {
 #pragma unroll
@@ -479,6 +498,10 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
     cp_async_wait<0>();
     __syncwarp();
 #undef VS
+    if constexpr (BWD) {  // fused gbsv: U x = y while the other resident matrices still factor
+        const bool wr = live && (!SKIPI || linfo == 0);
+        backsolve_group<KV, G, YSM>(n, ab, ldab, bv, ybuf_s, live, wr, t, (int)gbase);
+    }
     if (!live) return;
 
     // LAPACK's SET_FILLIN also zeroes fill-row positions whose matrix row is

@@ -26,15 +26,15 @@ __global__ void __launch_bounds__(128) gbtrf_generic_kernel(int m, int n, int kl
     const int warp = (int)((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
     const int lane = (int)lane_id();
     if (warp >= batch) return;
-    double *__restrict__ ab = A.get(warp);
-    int *__restrict__ ipiv = P.get(warp);
-    const int kv = kl + ku;
-    auto AB = [&](int r, int c) -> double & { return ab[(int64_t)c * ldab + r]; };
-
+    // quick return first: with m == 0 or n == 0 the pointer arrays may be NULL
     if (m == 0 || n == 0) {
         if (lane == 0) info[warp] = 0;
         return;
     }
+    double *__restrict__ ab = A.get(warp);
+    int *__restrict__ ipiv = P.get(warp);
+    const int kv = kl + ku;
+    auto AB = [&](int r, int c) -> double & { return ab[(int64_t)c * ldab + r]; };
     // initial fill-in zeroing, columns ku+1 .. min(kv,n)-1, rows kv-j .. kl-1
     for (int j = ku + 1; j <= min(kv, n) - 1; ++j)
         for (int r = kv - j + lane; r <= kl - 1; r += 32) AB(r, j) = 0.0;

@@ -109,6 +109,79 @@ def gen_rhs(n: int, nrhs: int, ldb: int | None = None, count: int = 1, first: in
     return out
 
 
+# ---- the same generator on a torch device (bitwise equal to gen_band / gen_rhs) ----
+# bench.py fills HBM-sized sweep batches on the GPU without a host round trip
+# (torch int64 arithmetic wraps modulo 2^64; logical shifts are masked).
+
+def _s64(u: int) -> int:
+    return u - (1 << 64) if u >= (1 << 63) else u
+
+
+def _mix_t(x):
+    import torch
+
+    def srl(v, s):
+        return (v >> s) & ((1 << (64 - s)) - 1)
+    x = x ^ srl(x, 30)
+    x = x * _s64(int(_M1))
+    x = x ^ srl(x, 27)
+    x = x * _s64(int(_M2))
+    x = x ^ srl(x, 31)
+    return x
+
+
+def _uniform_pm1_t(seed: int, stream: int, mat_idx, local):
+    import torch
+    key = _s64(int(_mix(np.array([(seed & 0xFFFFFFFF) | (stream << 32)], dtype=np.uint64))[0]))
+    ctr = (mat_idx << 32) ^ local
+    z = _mix_t(ctr * _s64(int(_GOLD)) + key)
+    u = ((z >> 11) & ((1 << 53) - 1)).to(torch.float64) * (1.0 / 9007199254740992.0)
+    return 2.0 * u - 1.0
+
+
+def gen_band_torch(m: int, n: int, kl: int, ku: int, count: int, first: int = 0, device="cpu",
+                   ldab: int | None = None, seed: int = SEED, sentinel: float = float("nan"), out=None):
+    """torch float64 [count, n, ldab] on `device`, bitwise equal to gen_band(...)."""
+    import torch
+    ldab = 2 * kl + ku + 1 if ldab is None else ldab
+    ldmin = 2 * kl + ku + 1
+    if out is None:
+        out = torch.empty((count, n, ldab), dtype=torch.float64, device=device)
+    out.fill_(sentinel)
+    mask = band_valid_mask(m, n, kl, ku, ldab)
+    cc, rr = np.nonzero(mask)
+    if cc.size == 0 or count == 0:
+        return out
+    flat = torch.from_numpy((cc * ldab + rr).astype(np.int64)).to(out.device)
+    local = torch.from_numpy((cc.astype(np.int64) * ldmin + rr)).to(out.device)[None, :]
+    view = out.view(count, n * ldab)
+    step = max(1, (1 << 24) // cc.size)
+    for s in range(0, count, step):
+        e = min(count, s + step)
+        idx = torch.arange(first + s, first + e, dtype=torch.int64, device=out.device)[:, None]
+        view[s:e].index_copy_(1, flat, _uniform_pm1_t(seed, _A_STREAM, idx, local))
+    return out
+
+
+def gen_rhs_torch(n: int, nrhs: int, count: int, first: int = 0, device="cpu", ldb: int | None = None,
+                  seed: int = SEED, sentinel: float = float("nan"), out=None):
+    """torch float64 [count, nrhs, ldb] on `device`, bitwise equal to gen_rhs(...)."""
+    import torch
+    ldb = max(1, n) if ldb is None else ldb
+    if out is None:
+        out = torch.empty((count, nrhs, ldb), dtype=torch.float64, device=device)
+    out.fill_(sentinel)
+    if n == 0 or nrhs == 0 or count == 0:
+        return out
+    local = torch.arange(nrhs * n, dtype=torch.int64, device=out.device)[None, :]
+    step = max(1, (1 << 24) // (nrhs * n))
+    for s in range(0, count, step):
+        e = min(count, s + step)
+        idx = torch.arange(first + s, first + e, dtype=torch.int64, device=out.device)[:, None]
+        out[s:e, :, :n] = _uniform_pm1_t(seed, _B_STREAM, idx, local).view(e - s, nrhs, n)
+    return out
+
+
 def shard_range(batch: int, rank: int, world: int) -> tuple[int, int]:
     """Contiguous shard [lo, hi) of rank r out of R."""
     return (batch * rank) // world, (batch * (rank + 1)) // world
@@ -137,6 +210,16 @@ def alg_bytes_fused(n: int, kl: int, ku: int, nrhs: int) -> tuple[int, int]:
     b_trf, _ = alg_bytes(n, n, kl, ku, nrhs)
     wu = sum(min(j, kv) + 1 for j in range(n))
     return b_trf + 16 * n * nrhs, 8 * wu + 16 * n * nrhs
+
+
+def alg_bytes_kind(n: int, kl: int, ku: int, nrhs: int, kind: str) -> int:
+    """Algorithmic HBM bytes per square matrix that ONE launch of the given class must
+    move (bandlu_trfs_plan byte classes): trf = B_trf; trf_fwd = B_trf + B in / y out;
+    trs_bwd = U entries + y in / x out; trs = B_trs; gbsv (the fused single launch) =
+    B_trf + B in / x out -- U is produced and consumed inside the kernel."""
+    b_trf, b_trs = alg_bytes(n, n, kl, ku, nrhs)
+    f_trf, f_bwd = alg_bytes_fused(n, kl, ku, nrhs)
+    return {"trf": b_trf, "trf_fwd": f_trf, "trs_bwd": f_bwd, "trs": b_trs, "gbsv": b_trf + 16 * n * nrhs}[kind]
 
 
 def nominal_flops(n: int, kl: int, ku: int, nrhs: int) -> tuple[int, int]:

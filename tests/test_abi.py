@@ -111,7 +111,7 @@ def test_variant_heuristic_is_shape_only(lib):
     assert b.trf_variant(512, 512, 10, 10) == b.ROWS
     assert b.rows_available(10, 10) and b.rows_available(2, 32) and b.rows_available(1, 1)
     assert not b.rows_available(0, 3) and not b.rows_available(3, 0)
-    assert b.tc_available(10, 10) and not b.tc_available(1, 1)  # opt-in tensor-core kernel
+    assert not b.tc_available(10, 10) and not b.thread_available(1, 1)  # opt-in builds only (-DBANDLU_WITH_TC/THREAD)
     assert b.trf_variant(256, 256, 1, 1) == b.ROWS  # thin bands: row-slot kernel too
     assert b.trf_variant(64, 64, 0, 3) == b.WINDOW
     assert b.trf_variant(100, 100, 32, 32) == b.ROWS  # kl+1 > 32 lanes: two-warp row-slot kernel
@@ -134,3 +134,22 @@ def test_product_package_does_not_import_oracle():
                 txt = open(os.path.join(dirpath, fn)).read()
                 assert "import oracle" not in txt and "from oracle" not in txt, fn
                 assert "bandlu_oracle" not in txt and "liboracle" not in txt, fn
+
+
+def test_trfs_plan_reports_the_launches(lib):
+    """bandlu_trfs_plan (no launch): the fused gbsv kernel for nrhs == 1 on row-slot
+    bands, forward-fused factorization + backward launch on other compiled bands,
+    trf + trs otherwise."""
+    from paper_conf_sc_abdelfattahtlad23_b200 import binding as b
+    p = b.trfs_plan(512, 10, 10, 1)
+    assert p == {"kernels": ["gbtrf_rows_kernel"], "bytes": ["gbsv"], "fused": True}
+    p = b.trfs_plan(512, 10, 10, 1, two_launch=True)
+    assert p["kernels"] == ["gbtrf_rows_kernel", "gbtrs_bwd_kernel"] and p["bytes"] == ["trf_fwd", "trs_bwd"]
+    p = b.trfs_plan(2048, 32, 32, 1)
+    assert p["kernels"] == ["gbtrf_wide_kernel", "gbtrs_window_kernel"] and not p["fused"]
+    p = b.trfs_plan(1024, 2, 32, 16)
+    assert p["kernels"] == ["gbtrf_rows_kernel", "gbtrs_window_kernel"] and p["bytes"] == ["trf", "trs"]
+    p = b.trfs_plan(100, 5, 9, 1)
+    assert p["kernels"] == ["gbtrf_generic_kernel", "gbtrs_generic_kernel"]
+    assert b.trfs_plan(0, 1, 1, 1)["kernels"] == []
+    assert lib.bandlu_trfs_plan(-1, 1, 1, 1, 0, None) < 0

@@ -34,3 +34,42 @@ def test_algorithmic_bytes_match_survey_table():
     assert I.alg_bytes(64, 64, 2, 2, 1) == (6252, 4760)              # C1
     assert I.alg_bytes(256, 256, 1, 1, 1) == (15316, 13280)          # C2
     assert I.alg_bytes(1024, 1024, 2, 32, 16) == (584892, 564560)    # C4
+
+
+def test_gpus_flag_self_launches_ranks():
+    """`bench.py --gpus 2` without a torchrun environment re-launches itself under
+    torch.distributed.run with 2 ranks (127.0.0.1); the reference arm runs on rank 0
+    only, so exactly one JSON line comes back, with n_gpus == 2 and the strong-scaling
+    global batch."""
+    env = {k: v for k, v in os.environ.items() if k not in ("RANK", "WORLD_SIZE", "LOCAL_RANK")}
+    r = subprocess.run([sys.executable, "bench.py", "--impl", "reference", "--gpus", "2", "--steps", "1",
+                        "--warmup", "3", "--config", "C1", "--scaling", "strong"], cwd=ROOT, capture_output=True,
+                       text=True, timeout=600, env=env)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["scaling"] == "strong" and d["config"]["global_batch"] == 100
+
+
+def test_gpus_flag_must_match_world_size():
+    env = dict(os.environ, WORLD_SIZE="1", RANK="0", LOCAL_RANK="0")
+    r = subprocess.run([sys.executable, "bench.py", "--gpus", "4", "--steps", "1"], cwd=ROOT, capture_output=True,
+                       text=True, timeout=300, env=env)
+    assert r.returncode == 2 and "WORLD_SIZE" in r.stderr
+
+
+def test_torch_generator_matches_numpy_generator():
+    """bench.py generates its HBM-sized inputs on the GPU with inputs.gen_band_torch;
+    it must reproduce the seeded generator bitwise (checked here on the CPU)."""
+    import numpy as np
+    sys.path.insert(0, ROOT)
+    from paper_conf_sc_abdelfattahtlad23_b200 import inputs as I
+    for m, n, kl, ku, ldab, first in [(64, 64, 2, 2, None, 0), (30, 20, 3, 2, 12, 7), (512, 512, 10, 10, None, 9999),
+                                      (40, 40, 32, 32, None, 2 ** 31 + 5)]:
+        a = I.gen_band(m, n, kl, ku, ldab=ldab, count=3, first=first)
+        b = I.gen_band_torch(m, n, kl, ku, count=3, first=first, ldab=ldab).numpy()
+        assert np.array_equal(np.isnan(a), np.isnan(b)) and np.array_equal(np.nan_to_num(a), np.nan_to_num(b))
+    r = I.gen_rhs(50, 3, ldb=53, count=4, first=99)
+    t = I.gen_rhs_torch(50, 3, count=4, first=99, ldb=53).numpy()
+    assert np.array_equal(np.isnan(r), np.isnan(t)) and np.array_equal(np.nan_to_num(r), np.nan_to_num(t))

@@ -389,3 +389,128 @@ def test_trf_batch_tail_after_other_launches(kl, ku):
         _check_trf(300, 300, kl, ku, batch=97, variant=variant)  # fills shared memory with live data
         for batch in (1, 3, 5):
             _check_trf(90, 90, kl, ku, batch=batch, variant=variant, first=batch)
+
+
+# ------------------------------------ the path bench.py times, at full batch
+# dgbtrfs (factorization + fused forward solve, then the backward launch) at
+# batches that select every matrices-per-warp instantiation of the backward
+# solve (bandlu.cu launch_trs_bwd_lean: 2 / 4 / 8 / 16 / 32), plus the C2 and
+# (32,32) backward kernels.  PAPER.md P:639-640, P:675-682 (backward solve).
+TRFS_FULL = [  # (batch, n, kl, ku)
+    (10000, 512, 10, 10),  # C3 exactly as bench.py times it
+    (5000, 512, 10, 10),
+    (20000, 64, 10, 10),
+    (40000, 40, 10, 7),
+    (3000, 200, 10, 10),
+    (10000, 50, 10, 10),   # PELE-like
+    (10000, 256, 1, 1),    # C2
+    (300, 2048, 32, 32),   # C5's widest band at its largest n
+    (1500, 1024, 2, 32),
+]
+
+
+def _sample_indices(batch, seed=7, per_warp=(2, 4, 8, 16, 32), extra=48):
+    """First and last matrix of the first, second, middle and last warp for each
+    matrices-per-warp grouping, plus random matrices (>= 64 in total)."""
+    idx = {0, batch - 1}
+    for g in per_warp:
+        warps = (batch + g - 1) // g
+        for w in (0, 1, warps // 2, warps - 1):
+            idx.update({min(batch - 1, w * g), min(batch - 1, w * g + g - 1)})
+    rng = np.random.default_rng(seed)
+    idx.update(int(i) for i in rng.integers(0, batch, extra))
+    return sorted(idx)
+
+
+@pytest.mark.parametrize("batch,n,kl,ku", TRFS_FULL)
+def test_trfs_full_batch_sampled_parity(batch, n, kl, ku):
+    A = torch.from_numpy(I.gen_band(n, n, kl, ku, count=batch)).cuda()
+    B = torch.from_numpy(I.gen_rhs(n, 1, count=batch)).cuda()
+    P = torch.zeros((batch, n), dtype=torch.int32, device="cuda")
+    info = torch.full((batch,), -7, dtype=torch.int32, device="cuda")
+    bl.dgbtrfs_strided_batched(n, kl, ku, A, P, B, info)
+    torch.cuda.synchronize()
+    sample = _sample_indices(batch)
+    assert len(sample) >= 64 or len(sample) == batch
+    sel = torch.tensor(sample, device="cuda")
+    Ag, Bg, Pg, Ig = (t.index_select(0, sel).cpu().numpy() for t in (A, B, P, info))
+    for k, i in enumerate(sample):
+        Ao = I.gen_band(n, n, kl, ku, count=1, first=i)
+        Bo = I.gen_rhs(n, 1, count=1, first=i)
+        ipo, info_o = oracle.dgbtrf(Ao, n, n, kl, ku)
+        oracle.dgbtrs(Ao, ipo, Bo, n, kl, ku)
+        assert Ig[k] == info_o[0], f"info of matrix {i}"
+        assert np.array_equal(Pg[k], ipo[0]), f"ipiv of matrix {i}"
+        assert np.all(same_bits(Ag[k], Ao[0])), f"factors of matrix {i}"
+        assert np.all(same_bits(Bg[k], Bo[0])), f"solution of matrix {i}"
+    j = torch.arange(n, device="cuda", dtype=torch.int32)
+    assert bool(torch.all(P >= j + 1)) and bool(torch.all(P <= torch.clamp(j + 1 + kl, max=n)))
+    assert int(info.abs().sum()) == 0
+
+
+# ------------------------------------------------ the fused gbsv kernel (f1)
+# One launch: factorization + forward substitution on the fly + backward
+# substitution by the same lanes (PAPER.md Sec. 7 P:686-702, generalised to any
+# n).  y(0..n-1) lives in shared memory when it fits (dgbsv may then leave B
+# untouched where info > 0), else in B (large n: dgbtrfs only; dgbsv takes two
+# launches).  Both plans must equal the oracle bitwise.
+FUSED_BANDS = [(10, 10), (10, 7), (2, 32), (1, 1), (2, 2), (2, 3), (4, 4)]
+
+
+def _trfs(A_np, B_np, n, kl, ku, phase=0):
+    Ag = torch.from_numpy(A_np).cuda(); Bg = torch.from_numpy(B_np).cuda()
+    batch = A_np.shape[0]
+    P = torch.zeros((batch, n), dtype=torch.int32, device="cuda")
+    inf = torch.full((batch,), -3, dtype=torch.int32, device="cuda")
+    bl.dgbtrfs_strided_batched(n, kl, ku, Ag, P, Bg, inf, phase=phase)
+    torch.cuda.synchronize()
+    return Ag.cpu().numpy(), P.cpu().numpy(), Bg.cpu().numpy(), inf.cpu().numpy()
+
+
+@pytest.mark.parametrize("kl,ku", FUSED_BANDS)
+@pytest.mark.parametrize("n", [3, 17, 130, 777, 1000])  # 777 / 1000: y beyond the shared-memory budget at (10,10)
+def test_fused_gbsv_kernel_vs_oracle_and_two_launch_plan(kl, ku, n):
+    plan = bl.trfs_plan(n, kl, ku, 1)
+    assert plan["fused"] and plan["kernels"] == ["gbtrf_rows_kernel"]
+    assert bl.trfs_plan(n, kl, ku, 1, two_launch=True)["kernels"][0] == "gbtrf_rows_kernel"
+    batch = 19  # ragged: not a multiple of matrices per warp / CTA
+    A = I.gen_band(n, n, kl, ku, count=batch, first=n)
+    B = I.gen_rhs(n, 1, ldb=n + 2, count=batch, first=n)
+    Ao, Bo = A.copy(), B.copy()
+    ipo, info_o = oracle.dgbtrf(Ao, n, n, kl, ku)
+    oracle.dgbtrs(Ao, ipo, Bo, n, kl, ku)
+    for phase in (0, bl.TRFS_TWO_LAUNCH):
+        Ag, Pg, Bg, Ig = _trfs(A.copy(), B.copy(), n, kl, ku, phase)
+        assert np.array_equal(Ig, info_o)
+        assert np.array_equal(Pg, ipo)
+        assert np.all(same_bits(Ag, Ao))
+        assert np.all(same_bits(Bg, Bo))  # incl. the NaN ldb padding rows
+
+
+@pytest.mark.parametrize("kl,ku", FUSED_BANDS)
+@pytest.mark.parametrize("n", [40, 512, 1000])
+def test_fused_dgbsv_leaves_b_untouched_where_singular(kl, ku, n):
+    """dgbsv through the fused kernel (y in shared memory; n = 1000 at (10,10)
+    takes the two-launch path): info / ipiv / factors / x bitwise, and B
+    bitwise unchanged for the matrices with a planted zero pivot (LAPACK DGBSV)."""
+    batch = 10
+    A = I.gen_band(n, n, kl, ku, count=batch)
+    kv = kl + ku
+    for b, z in ((2, 1), (5, n // 2), (9, n)):  # zero column z (1-based): info = z
+        A[b, z - 1, kl:kv + kl + 1] = np.where(np.isnan(A[b, z - 1, kl:kv + kl + 1]), np.nan, 0.0)
+    B = I.gen_rhs(n, 1, ldb=n + 1, count=batch)
+    Ao, Bo = A.copy(), B.copy()
+    ipo, info_o = oracle.dgbsv(Ao, Bo, n, kl, ku)
+    assert list(info_o[[2, 5, 9]]) == [1, n // 2, n]
+    Ag = torch.from_numpy(A).cuda(); Bg = torch.from_numpy(B).cuda()
+    P = torch.zeros((batch, n), dtype=torch.int32, device="cuda")
+    inf = torch.zeros(batch, dtype=torch.int32, device="cuda")
+    bl.dgbsv_strided_batched(n, kl, ku, Ag, P, Bg, inf)
+    torch.cuda.synchronize()
+    assert np.array_equal(inf.cpu().numpy(), info_o)
+    assert np.array_equal(P.cpu().numpy(), ipo)
+    assert np.all(same_bits(Ag.cpu().numpy(), Ao))
+    Bgn = Bg.cpu().numpy()
+    assert np.all(same_bits(Bgn, Bo))
+    for b in (2, 5, 9):
+        assert np.all(same_bits(Bgn[b], B[b]))

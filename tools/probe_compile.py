@@ -10,8 +10,8 @@ for kl,ku in pairs:
     else:
         lines.append('(void*)&gbtrs_window_kernel<%d,%d,Strided<const double>,Strided<const int>,Strided<double>>,'%(kl,ku))
 lines.append('};')
-open('paper_conf_sc_abdelfattahtlad23_b200/csrc/_probe.cu','w').write('\n'.join(lines)+'\n')
-r=subprocess.run('nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 --fmad=false -Xptxas -v -cubin -o /tmp/probe.cubin paper_conf_sc_abdelfattahtlad23_b200/csrc/_probe.cu',shell=True,capture_output=True,text=True)
+open('/tmp/_bandlu_probe.cu','w').write('\n'.join(lines)+'\n')
+r=subprocess.run('nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 --fmad=false -Xptxas -v -I paper_conf_sc_abdelfattahtlad23_b200/csrc -cubin -o /tmp/probe.cubin /tmp/_bandlu_probe.cu',shell=True,capture_output=True,text=True)
 for l in r.stderr.splitlines():
     if 'error' in l or 'Used' in l or 'spill' in l or 'Compiling' in l: print(l[:200])
 s=subprocess.run('cuobjdump -sass /tmp/probe.cubin',shell=True,capture_output=True,text=True).stdout
