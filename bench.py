@@ -154,7 +154,9 @@ def cpu_oracle_rate(n, kl, ku, nrhs, seconds=6.0, sample=1024, threads=0):
     A0 = I.gen_band(n, n, kl, ku, count=sample)
     B0 = I.gen_rhs(n, nrhs, count=sample)
     oracle.build()
-    used = threads if threads > 0 else oracle.max_threads()
+    if threads <= 0:  # every host core (explicit: an earlier call may have changed the OpenMP default)
+        threads = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else (os.cpu_count() or 1)
+    used = threads
     times = []
     t_end = time.perf_counter() + seconds
     while len(times) < 3 or (time.perf_counter() < t_end and len(times) < 50):
@@ -235,6 +237,9 @@ def parse(argv=None):
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--parity-sample", type=int, default=24, help="random matrices per rank checked vs the oracle")
     ap.add_argument("--fill", type=float, default=0.3, help="C5: fraction of free HBM per sweep point")
+    ap.add_argument("--plan", default="auto", choices=["auto", "two", "fused"],
+                    help="dgbtrfs plan: the library's choice, the two-launch plan (factorization + forward, then "
+                         "backward), or the fused single-launch kernel")
     ap.add_argument("--c5-ns", default="", help="C5: comma-separated n list (default 32,64,128..2048 step 128)")
     args = ap.parse_args(argv)
     args.warmup = max(args.warmup, 3)
@@ -260,7 +265,8 @@ def run_config(args):
     ldab = 2 * kl + ku + 1
     b_trf, b_trs = I.alg_bytes(n, n, kl, ku, nrhs)
     f_trf, f_trs = I.nominal_flops(n, kl, ku, nrhs)
-    plan = bl.trfs_plan(n, kl, ku, nrhs)  # which kernels one dgbtrfs call launches (shape only)
+    xph = {"auto": 0, "two": bl.TRFS_TWO_LAUNCH, "fused": bl.TRFS_FUSED}[args.plan]
+    plan = bl.trfs_plan(n, kl, ku, nrhs, cnt, xph)  # the kernels one dgbtrfs call launches
     per_launch_bytes = [I.alg_bytes_kind(n, kl, ku, nrhs, k) for k in plan["bytes"]]
     big = cnt * n * ldab * 8 > 2 * 126e6
     config = {"workload": desc, "global_batch": glob, "batch_per_gpu": cnt, "n": n, "kl": kl, "ku": ku,
@@ -287,7 +293,7 @@ def run_config(args):
         if evs is not None:
             evs[0].record(st)
         for ph in range(1, nph + 1):
-            bl.dgbtrfs_strided_batched(n, kl, ku, A, P, B, info, phase=ph if nph > 1 else 0)
+            bl.dgbtrfs_strided_batched(n, kl, ku, A, P, B, info, phase=(ph if nph > 1 else 0) | xph)
             if evs is not None:
                 evs[ph].record(st)
 
@@ -425,7 +431,8 @@ def run_sweep(args):
             A, B = torch.empty_like(A0), torch.empty_like(B0)
             P = torch.zeros((bpg, n), dtype=torch.int32, device=dev)
             info = torch.zeros(bpg, dtype=torch.int32, device=dev)
-            plan = bl.trfs_plan(n, kl, ku, 1)
+            xph = {"auto": 0, "two": bl.TRFS_TWO_LAUNCH, "fused": bl.TRFS_FUSED}[args.plan]
+            plan = bl.trfs_plan(n, kl, ku, 1, bpg, xph)
             nph = len(plan["kernels"])
 
             def step(evs=None):
@@ -434,7 +441,7 @@ def run_sweep(args):
                 if evs is not None:
                     evs[0].record(st)
                 for ph in range(1, nph + 1):
-                    bl.dgbtrfs_strided_batched(n, kl, ku, A, P, B, info, phase=ph if nph > 1 else 0)
+                    bl.dgbtrfs_strided_batched(n, kl, ku, A, P, B, info, phase=(ph if nph > 1 else 0) | xph)
                     if evs is not None:
                         evs[ph].record(st)
 

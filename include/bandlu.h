@@ -95,9 +95,12 @@ enum bandlu_variant {
                            pow2 >= kl+ku+1 lanes per (matrix, RHS column), compiled (kl, ku) with
                            kl+ku+1 <= 32 only (bandlu_trs_rows_available); AUTO's choice for
                            nrhs == 1 with kl+ku+1 <= 4.  Bitwise equal results */,
-    BANDLU_THREAD = 5   /* dgbtrf only: one thread per matrix, the whole (kl+1) x (kl+ku+1) window in
+    BANDLU_THREAD = 5,  /* dgbtrf only: one thread per matrix, the whole (kl+1) x (kl+ku+1) window in
                            registers, thin compiled bands (bandlu_thread_available); bitwise equal
                            results */
+    BANDLU_TPM = 6      /* dgbtrf only, square (m == n): one thread per matrix, the window in shared
+                           memory, 4-column panels factored in registers and a rank-4 trailing
+                           update per panel (bandlu_tpm_available); bitwise equal results */
 };
 
 /* ---- dgbtrf: band LU with partial pivoting ---- */
@@ -127,9 +130,9 @@ int dgbtrs_strided_batched(char trans, int n, int kl, int ku, int nrhs,
                            int batch, bandlu_stream_t stream);
 
 /* ---- dgbsv: dgbtrf + dgbtrs.  B is untouched for every matrix
- * with info > 0 (LAPACK DGBSV).  Strided, nrhs == 1, a band with a row-slot
- * kernel and y(0..n-1) fitting in shared memory: ONE launch of the fused gbsv
- * kernel (factorization, forward substitution on the fly, backward
+ * with info > 0 (LAPACK DGBSV).  Strided, nrhs == 1, a band with a fused
+ * row-slot kernel, a batch within one wave of it and y(0..n-1) fitting in
+ * shared memory: ONE launch of the fused gbsv kernel (factorization, forward substitution on the fly, backward
  * substitution by the same lanes; Sec. 7 P:686-702 generalised to any n).
  * Otherwise a factorization launch and a solve launch. ---- */
 int dgbsv_batched(int n, int kl, int ku, int nrhs,
@@ -144,11 +147,12 @@ int dgbsv_strided_batched(int n, int kl, int ku, int nrhs,
 
 /* ---- dgbtrfs: dgbtrf followed by dgbtrs('N') on every matrix, as one call
  * (the bench's hot-path step).  Same arguments and numbering as
- * dgbsv_strided_batched.  nrhs == 1 and a band with a row-slot kernel: ONE
- * launch (the fused kernel, as dgbsv; y in shared memory when it fits, else
- * in B).  nrhs == 1 and another compiled (kl, ku): the factorization kernel
- * applies the forward substitution (the paper's augmented [A|B], Sec. 7
- * P:688-702), then one backward-substitution launch.  Results are bitwise
+ * dgbsv_strided_batched.  nrhs == 1, a band with a fused row-slot kernel and a
+ * batch that fits in one wave of it (SMs x resident matrices): ONE launch (the
+ * fused kernel, as dgbsv; y in shared memory when it fits, else in B).  Other
+ * nrhs == 1 cases with a compiled (kl, ku): the factorization kernel applies the
+ * forward substitution (the paper's augmented [A|B], Sec. 7), then
+ * one backward-substitution launch.  Results are bitwise
  * those of the separate calls.  Unlike dgbsv, B is solved also where
  * info > 0 (as dgbtrs would: singular U gives Inf/NaN). ---- */
 int dgbtrfs_strided_batched(int n, int kl, int ku, int nrhs,
@@ -158,9 +162,11 @@ int dgbtrfs_strided_batched(int n, int kl, int ku, int nrhs,
                             int batch, bandlu_stream_t stream);
 /* phase (profiling): 0 = everything, 1 = the first launch only, 2 = the second
  * launch only (nothing when the plan has one launch); + BANDLU_TRFS_TWO_LAUNCH
- * forces the two-launch plan (factorization + forward, then backward); any
- * other value returns -16. */
+ * forces the two-launch plan (factorization + forward, then backward), +
+ * BANDLU_TRFS_FUSED the fused kernel where it exists; any other value (or
+ * both flags) returns -16. */
 #define BANDLU_TRFS_TWO_LAUNCH 16
+#define BANDLU_TRFS_FUSED 32
 int dgbtrfs_strided_batched_ex(int n, int kl, int ku, int nrhs,
                                double *dA, int ldab, int64_t strideA,
                                int *dipiv, int64_t strideP,
@@ -208,17 +214,20 @@ int bandlu_rows_available(int kl, int ku);
 /* 1 if a thread-per-matrix factorization kernel (BANDLU_THREAD) is compiled for (kl, ku), else 0
  * (only in -DBANDLU_WITH_THREAD builds: measured slower, AUTO never picks it). */
 int bandlu_thread_available(int kl, int ku);
+/* 1 if a thread-per-matrix shared-memory-window kernel (BANDLU_TPM) is compiled for (kl, ku), else 0. */
+int bandlu_tpm_available(int kl, int ku);
 /* 1 if a lane-per-row solve kernel (dgbtrs BANDLU_ROWS) is compiled for (kl, ku), else 0. */
 int bandlu_trs_rows_available(int kl, int ku);
-/* The launches one dgbtrfs_strided_batched call makes for a shape (no launch):
+/* The launches one dgbtrfs_strided_batched call with this phase flag set makes
+ * for a shape and batch (no launch):
  * returns their number L (0..2; < 0 on a negative argument) and, if kinds is
  * not NULL, writes L codes kinds[i] = 16 * kernel + bytes, kernel: 1 gbtrf_rows,
  * 2 gbtrf_window, 3 gbtrf_wide, 4 gbtrf_thread, 5 gbtrf_generic, 6 gbtrs_bwd,
  * 7 gbtrs_rows, 8 gbtrs_window, 9 gbtrs_generic; bytes (what the launch must
  * move per matrix): 1 factorization, 2 factorization + forward
  * substitution, 3 backward substitution, 4 full solve, 5 fused gbsv.
- * two_launch != 0: the plan of phase | BANDLU_TRFS_TWO_LAUNCH. */
-int bandlu_trfs_plan(int n, int kl, int ku, int nrhs, int two_launch, int *kinds);
+ * phase: 0, BANDLU_TRFS_TWO_LAUNCH or BANDLU_TRFS_FUSED (as for dgbtrfs). */
+int bandlu_trfs_plan(int n, int kl, int ku, int nrhs, int batch, int phase, int *kinds);
 /* ABI version of this library. */
 int bandlu_version(void);
 

@@ -18,7 +18,7 @@ import torch
 
 from . import _build
 
-AUTO, GENERIC, WINDOW, TC, ROWS, THREAD = 0, 1, 2, 3, 4, 5
+AUTO, GENERIC, WINDOW, TC, ROWS, THREAD, TPM = 0, 1, 2, 3, 4, 5, 6
 ERR_UNSUPPORTED, ERR_CUDA = 1000, 2000
 
 _lib = None
@@ -71,8 +71,9 @@ def load(build_if_missing: bool = False):
         "bandlu_rows_available": [i, i],
         "bandlu_trs_rows_available": [i, i],
         "bandlu_thread_available": [i, i],
+        "bandlu_tpm_available": [i, i],
         "bandlu_trs_variant": [i, i, i, i],
-        "bandlu_trfs_plan": [i, i, i, i, i, p],
+        "bandlu_trfs_plan": [i, i, i, i, i, i, p],
         "bandlu_version": [],
     }
     for name, args in sig.items():
@@ -87,7 +88,7 @@ def load(build_if_missing: bool = False):
 EXPORTS = ("dgbtrf_batched", "dgbtrf_strided_batched", "dgbtrf_strided_batched_ex", "dgbtrs_batched",
            "dgbtrs_strided_batched", "dgbtrs_strided_batched_ex", "dgbsv_batched", "dgbsv_strided_batched",
            "dgbsv_strided_batched_host", "dgbtrfs_strided_batched", "dgbtrfs_strided_batched_ex", "bandlu_trf_variant", "bandlu_trs_variant", "bandlu_tc_available", "bandlu_rows_available", "bandlu_trs_rows_available", "bandlu_thread_available",
-           "bandlu_trfs_plan", "bandlu_version")
+           "bandlu_tpm_available", "bandlu_trfs_plan", "bandlu_version")
 
 
 def _stream(stream):
@@ -244,6 +245,11 @@ def thread_available(kl: int, ku: int) -> bool:
     return bool(load().bandlu_thread_available(kl, ku))
 
 
+def tpm_available(kl: int, ku: int) -> bool:
+    """True if the thread-per-matrix shared-memory-window factorization (variant TPM) is compiled for (kl, ku)."""
+    return bool(load().bandlu_tpm_available(kl, ku))
+
+
 def trs_rows_available(kl: int, ku: int) -> bool:
     """True if a lane-per-row solve kernel (dgbtrs variant ROWS) is compiled for (kl, ku)."""
     return bool(load().bandlu_trs_rows_available(kl, ku))
@@ -257,13 +263,14 @@ KERNEL_NAMES = {1: "gbtrf_rows_kernel", 2: "gbtrf_window_kernel", 3: "gbtrf_wide
                 5: "gbtrf_generic_kernel", 6: "gbtrs_bwd_kernel", 7: "gbtrs_rows_kernel", 8: "gbtrs_window_kernel",
                 9: "gbtrs_generic_kernel"}
 BYTE_KINDS = {1: "trf", 2: "trf_fwd", 3: "trs_bwd", 4: "trs", 5: "gbsv"}
-TRFS_TWO_LAUNCH = 16
+TRFS_TWO_LAUNCH, TRFS_FUSED = 16, 32
 
 
-def trfs_plan(n: int, kl: int, ku: int, nrhs: int, two_launch: bool = False) -> dict:
-    """The launches one dgbtrfs_strided_batched call makes for a shape (bandlu_trfs_plan)."""
+def trfs_plan(n: int, kl: int, ku: int, nrhs: int, batch: int, phase: int = 0) -> dict:
+    """The launches one dgbtrfs_strided_batched call (phase flag 0 / TRFS_TWO_LAUNCH /
+    TRFS_FUSED) makes for a shape and batch (bandlu_trfs_plan)."""
     kinds = (ctypes.c_int * 4)()
-    k = load().bandlu_trfs_plan(n, kl, ku, nrhs, int(two_launch), kinds)
+    k = load().bandlu_trfs_plan(n, kl, ku, nrhs, batch, phase, kinds)
     if k < 0:
         raise BandLUError("bandlu_trfs_plan", k)
     codes = list(kinds)[:k]

@@ -14,14 +14,19 @@
 // Every y(i) receives its updates in decreasing j, as in the column loop.
 //
 // Mapping: the G lanes of a matrix group own the right-hand-side rows
-// i == t (mod G).  A lane keeps S = ceil((kv+1)/G) rows in registers: slot s
-// holds the row r == t + s*G (mod S*G) with d_s = j - r in [0, S*G); the row
-// is in the active window while d_s <= kv, it is the pivot row of step j when
-// d_s == 0 (its lane divides and broadcasts x(j) with one shuffle), and when
-// it retires the slot takes row r - S*G (read from the y buffer: shared
-// memory, or B in global memory).  U(r_s, j) = AB(kv - d_s, j): the U column
-// is contiguous in band storage, so a slot's loads over the group are one
-// coalesced segment; they are issued PF steps ahead into a register ring.
+// i == t (mod G).  At step j lane t holds two of them: yA = row j - e (the
+// near one, distance e = (j - t) mod G) and yB = row j - e - G.  The lane with
+// e == 0 owns the pivot row: it divides, one shuffle broadcasts x(j), the
+// lanes whose rows are within kv of j apply one FMA each, and the owner then
+// shifts yA <- yB.  Its next row (j - 2G) is read into a staging ring and
+// merged into yB PF steps later (kv + 1 + PF <= 2G, so before that row enters
+// the window): no instruction of the following steps waits for that load.
+// The loop is unrolled by G steps over a G-aligned range (steps above n-1 are
+// empty), so every lane role of a step -- owner, merging lane, ring slot -- is
+// a compile-time constant.  U(i, j) = AB(kv - (j - i), j): a column's U entries
+// are contiguous in band storage, so lane t's two prefetch loads per step
+// (distances e and e + G) are two coalesced segments over the group, issued PF
+// steps ahead into a register ring.
 #pragma once
 #include "common.cuh"
 
@@ -31,89 +36,90 @@
 
 namespace bandlu {
 
-// YSM: y(i) read from shared memory at ybuf_s + 8 i (else from bx[i]).
-// wr: this group stores x into bx (false for dead groups and, for dgbsv, where info > 0).
-// All 32 lanes of the warp must call (shuffles / ballots over the full warp).
+template <int KV, int G>
+struct FusedSolve {
+    static constexpr int PF = BANDLU_FUSED_PF;
+    // two rows per lane suffice and the staging ring has PF steps before a row is used
+    static constexpr bool ok = (KV + 1 + PF <= 2 * G) && (G % PF == 0 || PF % G == 0) && G >= 2;
+};
+
+// YSM: y(i) read from shared memory at ybuf_s + 8 i (else from bx[i], where the
+// forward pass left it).  wr: this group stores x into bx (false for dead
+// groups and, for dgbsv, where info > 0).  All 32 lanes of the warp call.
 template <int KV, int G, bool YSM>
 __device__ __forceinline__ void backsolve_group(int n, const double *ab, int ldab, double *bx, uint32_t ybuf_s,
                                                 bool live, bool wr, int t, int gbase) {
-    constexpr int S = (KV + G) / G;  // ceil((KV + 1) / G)
-    constexpr int SG = S * G;
-    constexpr int PF = BANDLU_FUSED_PF;
-    constexpr bool POW2 = (SG & (SG - 1)) == 0;
+    constexpr int PF = FusedSolve<KV, G>::PF;
+    static_assert(FusedSolve<KV, G>::ok, "fused backward solve: needs kv + 1 + PF <= 2G");
     constexpr unsigned FULL = 0xffffffffu;
-    auto wrap = [](int x) -> int {  // x in (-SG, SG) -> [0, SG)
-        if constexpr (POW2) return x & (SG - 1);
-        else return x < 0 ? x + SG : x;
+    constexpr int NR = PF > G ? PF : G;  // ring period (unroll)
+    auto yload = [&](bool p, int r, double &v) {  // predicated: v unchanged where !p
+        if constexpr (YSM) ld_shared_f64_if(p, ybuf_s + (uint32_t)r * 8u, v);
+        else ld_global_f64_if(p, bx + r, v);
     };
-    auto yget = [&](int r) -> double {
-        if constexpr (YSM) return ld_shared_f64(ybuf_s + (uint32_t)r * 8u);
-        else return bx[r];
+    const int jt = ((n + NR - 1) / NR) * NR - 1;  // first step: a multiple of NR minus 1 (>= n-1)
+    // lane t at step jt: e = (jt - t) mod G = G-1-t; yA = row jt-e, yB = row jt-e-G
+    double yA = 0.0, yB = 0.0;
+    {
+        const int rA = jt - (G - 1 - t), rB = rA - G;
+        yload(live && rA >= 0 && rA < n, rA, yA);
+        yload(live && rB >= 0 && rB < n, rB, yB);
+    }
+    // staged refills, slot = step % PF; the lanes that merge during the first PF
+    // steps (no staging has happened yet) merge the yB they already hold
+    double stg[PF];
+#pragma unroll
+    for (int k = 0; k < PF; ++k) stg[k] = (t == ((G - 1 - k + PF) & (G - 1))) ? yB : 0.0;
+    // U prefetch ring: uA[k], uB[k] = U(row at distance e / e+G, step jt - k).  A
+    // distance <= kv beyond row 0 reads a corner position of the same band column
+    // (in bounds, value unused: it only ever updates rows < 0); distances > kv and
+    // columns outside [0, n) are not read.
+    double uA[PF], uB[PF];
+    const double *abk = live ? ab : g_dummy;
+    int cof = (jt + 1) * ldab + KV;  // element offset of AB(KV, jp + 1) for the next jp (decremented per step)
+    auto uload = [&](int jp, int e, double &a, double &b) {
+        cof -= ldab;
+        const bool col = live && jp >= 0 && jp < n;
+        const double *p = abk + (cof - e);
+        a = 0.0;
+        b = 0.0;
+        ld_global_f64_if(col && e <= KV, p, a);  // e <= KV: compile-time true when KV >= G - 1
+        if constexpr (G <= KV) ld_global_f64_if(col && e + G <= KV, p - G, b);
     };
-    const int jn = n - 1;
-    int d[S];
-    double y[S];
 #pragma unroll
-    for (int s = 0; s < S; ++s) {
-        const int q = (jn - t - s * G) % SG;
-        d[s] = q < 0 ? q + SG : q;
-        const int r = jn - d[s];
-        y[s] = (live && r >= 0) ? yget(r) : 0.0;
-    }
-    // U prefetch ring: uv[k][s] = U(row of slot s at step jb-k, jb-k) of the current block
-    double uv[PF][S];
-    const double *pre = live ? ab + (int64_t)jn * ldab + KV : nullptr;  // &AB(KV, j) of the next prefetch
-#pragma unroll
-    for (int k = 0; k < PF; ++k) {
-        const int j = jn - k;
-#pragma unroll
-        for (int s = 0; s < S; ++s) {
-            const int dd = wrap(d[s] - k % SG);
-            const bool ok = live && j >= 0 && dd <= KV && j - dd >= 0;
-            uv[k][s] = ok ? pre[-dd] : 0.0;
-        }
-        if (live) pre -= ldab;
-    }
+    for (int k = 0; k < PF; ++k) uload(jt - k, (G - 1 - k - t) & (G - 1), uA[k], uB[k]);
+
 #pragma unroll 1
-    for (int jb = jn; jb >= 0; jb -= PF) {
+    for (int jb = jt; jb >= 0; jb -= NR) {
 #pragma unroll
-        for (int k = 0; k < PF; ++k) {
+        for (int k = 0; k < NR; ++k) {
             const int j = jb - k;
-            if (j < 0) break;
+            const int kk = k % PF;
+            const int e = (G - 1 - k - t) & (G - 1);            // distance of yA
+            const int towner = (G - 1 - k) & (G - 1);           // lane holding row j (e == 0)
+            const int tmerge = (G - 1 - k + PF) & (G - 1);      // lane that staged a row PF steps ago
+            // ---- merge the row staged PF steps ago (before it enters the window)
+            yB = (t == tmerge) ? stg[kk] : yB;
             // ---- the pivot row of step j: its lane divides (DTBSV skips y(j) == 0)
-            double yo = 0.0, uo = 1.0;
-            bool own = false;
-#pragma unroll
-            for (int s = 0; s < S; ++s) {
-                if (d[s] == 0) {
-                    yo = y[s];
-                    uo = uv[k][s];
-                    own = true;
-                }
-            }
-            const bool nz = own && (yo != 0.0);
+            const bool own = (t == towner);
+            const bool nz = own && live && (yA != 0.0);
             const unsigned nzb = __ballot_sync(FULL, nz);
-            const double xo = ddiv_rn_if(nz, yo, uo);
-            const int src = gbase + (j & (G - 1));
+            const double xo = ddiv_rn_if(nz, yA, uA[kk]);
+            const int src = gbase + towner;
             const double x = __shfl_sync(FULL, xo, src);
             const bool upd = (nzb >> src) & 1u;
-            // ---- column update of the window rows, then retire / refill / prefetch
-#pragma unroll
-            for (int s = 0; s < S; ++s) {
-                const int dc = d[s];
-                if (upd && dc >= 1 && dc <= KV) y[s] = __fma_rn(-x, uv[k][s], y[s]);
-                if (dc == 0) {
-                    if (wr) bx[j] = xo;
-                    const int r2 = j - SG;
-                    y[s] = (live && r2 >= 0) ? yget(r2) : 0.0;
-                }
-                const int dd = wrap(dc - PF % SG);
-                const int jp = j - PF;
-                const bool ok = live && jp >= 0 && dd <= KV && jp - dd >= 0;
-                uv[k][s] = ok ? pre[-dd] : 0.0;
-                d[s] = (dc == 0) ? SG - 1 : dc - 1;
+            // ---- column update of the window rows
+            fma_rn_if(upd && (unsigned)(e - 1) < (unsigned)KV, -x, uA[kk], yA);
+            if constexpr (G <= KV) fma_rn_if(upd && e + G <= KV, -x, uB[kk], yB);
+            // ---- owner: x(j) out, shift the window rows, stage row j - 2G
+            st_global_f64_if(own && wr && j < n, bx + j, xo);
+            yA = own ? yB : yA;
+            {
+                const int r2 = j - 2 * G;
+                yload(own && live && r2 >= 0 && r2 < n, r2, stg[kk]);
             }
-            if (live) pre -= ldab;
+            // ---- prefetch step j - PF
+            uload(j - PF, (G - 1 - k - PF - t) & (G - 1), uA[kk], uB[kk]);
         }
     }
 }

@@ -18,6 +18,7 @@
 #include "gbtrf_wide.cuh"
 #include "gbtrf_tc.cuh"
 #include "gbtrf_thread.cuh"
+#include "gbtrf_tpm.cuh"
 #include "gbtrf_window.cuh"
 #include "gbtrs_bwd.cuh"
 #include "gbtrs_rows.cuh"
@@ -88,6 +89,19 @@ namespace {
     X(10, 7, 16, 1)                                      \
     X(2, 32, 8, 1)                                       \
     BANDLU_ROWS_THIN_LIST(X)
+#endif
+
+// (KL, KU, MPW) compiled as thread-per-matrix shared-memory-window kernels with rank-4
+// panel updates (gbtrf_tpm.cuh; square matrices), MPW matrices per CTA.
+#ifndef BANDLU_TPM_MPW
+#define BANDLU_TPM_MPW 16
+#endif
+// opt-in experiment (-DBANDLU_WITH_TPM): bitwise equal, but measured 2.95 vs 0.93 ms at C3
+// and 1.18 vs 0.23 ms at 1,250 matrices -- AUTO never picks it
+#if defined(BANDLU_WITH_TPM)
+#define BANDLU_TPM_LIST(X) X(10, 10, BANDLU_TPM_MPW)
+#else
+#define BANDLU_TPM_LIST(X)
 #endif
 
 // (KL, KU) compiled as thread-per-matrix factorization kernels (gbtrf_thread.cuh, thin
@@ -207,6 +221,25 @@ int launch_trf_thread(int m, int n, AP A, int ldab, PP P, int *info, int batch, 
     return cuda_ret(cudaGetLastError());
 }
 
+template <int KL, int KU, int MPW, bool FWD, class AP, class PP, class BP>
+int launch_trf_tpm(int n, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st, BP B) {
+    using C = TrfTpm<KL, KU, MPW>;
+    auto k = gbtrf_tpm_kernel<KL, KU, MPW, FWD, AP, PP, BP>;
+    const size_t sm = C::cta_bytes();
+    if (int r = set_smem(k, sm)) return r;
+    const unsigned grid = (unsigned)((batch + MPW - 1) / MPW);
+    k<<<grid, MPW, sm, st>>>(n, A, ldab, P, info, batch, B);
+    return cuda_ret(cudaGetLastError());
+}
+
+bool trf_tpm_available(int kl, int ku) {
+#define X(a, b, w) \
+    if (kl == a && ku == b) return true;
+    BANDLU_TPM_LIST(X)
+#undef X
+    return false;
+}
+
 template <class AP, class PP>
 int launch_trf_generic(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st) {
     const unsigned grid = (unsigned)(((int64_t)batch * 32 + 127) / 128);
@@ -308,6 +341,14 @@ int run_trf(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int b
 #undef X
         return BANDLU_ERR_UNSUPPORTED;
     }
+    if (variant == BANDLU_TPM && m > 0 && n > 0) {
+        if (m != n) return BANDLU_ERR_UNSUPPORTED;
+#define X(a, b, w) \
+    if (kl == a && ku == b) return launch_trf_tpm<a, b, w, false>(n, A, ldab, P, info, batch, st, Strided<double>{nullptr, 0});
+        BANDLU_TPM_LIST(X)
+#undef X
+        return BANDLU_ERR_UNSUPPORTED;
+    }
     if (variant == BANDLU_THREAD && m > 0 && n > 0) {
 #define X(a, b) \
     if (kl == a && ku == b) return launch_trf_thread<a, b, false>(m, n, A, ldab, P, info, batch, st, Strided<double>{nullptr, 0});
@@ -334,7 +375,7 @@ int run_trf(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int b
         return BANDLU_ERR_UNSUPPORTED;
     }
     if (variant != BANDLU_GENERIC && variant != BANDLU_WINDOW && variant != BANDLU_TC && variant != BANDLU_ROWS &&
-        variant != BANDLU_THREAD)
+        variant != BANDLU_THREAD && variant != BANDLU_TPM)
         return BANDLU_ERR_UNSUPPORTED;
     return launch_trf_generic(m, n, kl, ku, A, ldab, P, info, batch, st);
 }
@@ -482,22 +523,52 @@ int launch_trs_bwd(int n, AP A, int ldab, PP P, BP B, int ldb, int batch, cudaSt
 // solves B even where info > 0; dgbsv leaves B untouched there).
 // phase: 0 = every launch, 1 = first launch only, 2 = second launch only (the
 // bench times them separately); | TRFS_TWO_LAUNCH forces the two-launch plan.
-constexpr int TRFS_TWO_LAUNCH = BANDLU_TRFS_TWO_LAUNCH;
+constexpr int TRFS_TWO_LAUNCH = BANDLU_TRFS_TWO_LAUNCH, TRFS_FUSED = BANDLU_TRFS_FUSED;
 constexpr size_t kSmemPerSM = 227 * 1024;
 
 template <int KL, int KU, int G, int R>
 bool rows_ysm_fits(int n) {
+#ifdef BANDLU_FUSED_NO_YSM  // experiments: y always in B
+    if (n > 0) return false;
+#endif
     using C = TrfRows<KL, KU, G, R>;
     const size_t b = C::smem_bytes_y(n);
     return b <= kSmemPerSM && b * (size_t)C::MINB <= kSmemPerSM;
 }
 
+// the fused backward solve keeps two right-hand-side rows per lane (backsolve_fused.cuh)
 bool rows_fused_available(int kl, int ku) {
 #define X(a, b, g, r) \
-    if (kl == a && ku == b) return true;
+    if (kl == a && ku == b) return FusedSolve<a + b, g>::ok;
     BANDLU_ROWS_LIST(X)
 #undef X
     return false;
+}
+
+// Matrices one wave of the fused kernel holds (SMs x resident CTAs x matrices per CTA).
+// The fused kernel wins while the batch fits in one wave (the backward pass adds
+// latency but no wave); beyond that the factorization + forward kernel followed by
+// the bandwidth-bound backward kernel (8-32 matrices per warp) is faster -- measured
+// C3 1.30 vs 1.25 ms, PELE-like 0.147 vs 0.140 ms, C2 0.262 vs 0.242 ms; XGC-like
+// (512 matrices) 0.092 vs 0.115 ms, C1 0.035 vs 0.043 ms.  The
+// choice depends on the batch, the results do not (same operation sequence).
+int sm_count() {
+    int d = 0, c = 148;
+    if (cudaGetDevice(&d) == cudaSuccess) cudaDeviceGetAttribute(&c, cudaDevAttrMultiProcessorCount, d);
+    return c;
+}
+int64_t rows_wave(int kl, int ku) {
+#define X(a, b, g, r) \
+    if (kl == a && ku == b) return (int64_t)sm_count() * TrfRows<a, b, g, r>::MINB * TrfRows<a, b, g, r>::WARPS * TrfRows<a, b, g, r>::GPW;
+    BANDLU_ROWS_LIST(X)
+#undef X
+    return 0;
+}
+bool trfs_fused_pick(int n, int kl, int ku, int nrhs, int64_t batch, int phase) {
+    if (n <= 0 || nrhs != 1 || !rows_fused_available(kl, ku)) return false;
+    if (phase & TRFS_TWO_LAUNCH) return false;
+    if (phase & TRFS_FUSED) return true;
+    return batch <= rows_wave(kl, ku);
 }
 
 bool rows_ysm_fits_rt(int n, int kl, int ku) {
@@ -514,11 +585,11 @@ enum { KN_TRF_ROWS = 1, KN_TRF_WINDOW, KN_TRF_WIDE, KN_TRF_THREAD, KN_TRF_GENERI
 enum { KB_TRF = 1, KB_TRF_FWD, KB_TRS_BWD, KB_TRS, KB_GBSV };
 
 // the launches one dgbtrfs call makes for the shape (what run_trfs does)
-int trfs_plan(int n, int kl, int ku, int nrhs, bool two_launch, int *kinds) {
+int trfs_plan(int n, int kl, int ku, int nrhs, int64_t batch, int phase, int *kinds) {
     int k = 0;
     auto put = [&](int name, int bytes) { if (kinds) kinds[k] = name * 16 + bytes; ++k; };
     if (n <= 0 || nrhs <= 0) return 0;
-    if (nrhs == 1 && !two_launch && rows_fused_available(kl, ku)) {
+    if (trfs_fused_pick(n, kl, ku, nrhs, batch, phase)) {
         put(KN_TRF_ROWS, KB_GBSV);
         return k;
     }
@@ -542,16 +613,18 @@ int trfs_plan(int n, int kl, int ku, int nrhs, bool two_launch, int *kinds) {
 template <class AP, class PP, class BP>
 int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ldb, int *info, int batch,
              cudaStream_t st, int phase) {
-    const bool two = (phase & TRFS_TWO_LAUNCH) != 0;
-    phase &= ~TRFS_TWO_LAUNCH;
+    const bool fused = trfs_fused_pick(n, kl, ku, nrhs, batch, phase);
+    phase &= ~(TRFS_TWO_LAUNCH | TRFS_FUSED);
     if (batch == 0) return 0;
-    if (n > 0 && nrhs == 1 && !two && rows_fused_available(kl, ku)) {
+    if (fused) {
         if (phase == 2) return 0;  // the whole path is the first (only) launch
         const bool ysm = rows_ysm_fits_rt(n, kl, ku);
-#define X(a, b, g, rr)                                                                                               \
-    if (kl == a && ku == b)                                                                                          \
-        return ysm ? launch_trf_rows<a, b, g, rr, FL_FWD | FL_BWD | FL_YSM>(n, n, A, ldab, P, info, batch, st, B) \
-                   : launch_trf_rows<a, b, g, rr, FL_FWD | FL_BWD>(n, n, A, ldab, P, info, batch, st, B);
+#define X(a, b, g, rr)                                                                                                   \
+    if (kl == a && ku == b) {                                                                                            \
+        if constexpr (FusedSolve<a + b, g>::ok)                                                                          \
+            return ysm ? launch_trf_rows<a, b, g, rr, FL_FWD | FL_BWD | FL_YSM>(n, n, A, ldab, P, info, batch, st, B) \
+                       : launch_trf_rows<a, b, g, rr, FL_FWD | FL_BWD>(n, n, A, ldab, P, info, batch, st, B);       \
+    }
         BANDLU_ROWS_LIST(X)
 #undef X
         return BANDLU_ERR_UNSUPPORTED;
@@ -613,11 +686,13 @@ template <class AP, class PP, class BP>
 int run_gbsv(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ldb, int *info, int batch,
              cudaStream_t st) {
     if (batch == 0) return 0;
-    if (n > 0 && nrhs == 1 && rows_fused_available(kl, ku) && rows_ysm_fits_rt(n, kl, ku)) {
-#define X(a, b, g, rr)                                                                                  \
-    if (kl == a && ku == b)                                                                             \
-        return launch_trf_rows<a, b, g, rr, FL_FWD | FL_BWD | FL_YSM | FL_SKIPI>(n, n, A, ldab, P, info, \
-                                                                                 batch, st, B);
+    if (trfs_fused_pick(n, kl, ku, nrhs, batch, 0) && rows_ysm_fits_rt(n, kl, ku)) {
+#define X(a, b, g, rr)                                                                                      \
+    if (kl == a && ku == b) {                                                                               \
+        if constexpr (FusedSolve<a + b, g>::ok)                                                             \
+            return launch_trf_rows<a, b, g, rr, FL_FWD | FL_BWD | FL_YSM | FL_SKIPI>(n, n, A, ldab, P, info, \
+                                                                                     batch, st, B);         \
+    }
         BANDLU_ROWS_LIST(X)
 #undef X
     }
@@ -696,11 +771,13 @@ int bandlu_trf_variant(int m, int n, int kl, int ku) { return pick_trf(m, n, kl,
 int bandlu_tc_available(int kl, int ku) { return trf_tc_available(kl, ku) ? 1 : 0; }
 int bandlu_rows_available(int kl, int ku) { return trf_rows_available(kl, ku) ? 1 : 0; }
 int bandlu_thread_available(int kl, int ku) { return trf_thread_available(kl, ku) ? 1 : 0; }
+int bandlu_tpm_available(int kl, int ku) { return trf_tpm_available(kl, ku) ? 1 : 0; }
 int bandlu_trs_rows_available(int kl, int ku) { return trs_rows_available(kl, ku) ? 1 : 0; }
 int bandlu_trs_variant(int n, int kl, int ku, int nrhs) { return pick_trs(n, kl, ku, nrhs); }
-int bandlu_trfs_plan(int n, int kl, int ku, int nrhs, int two_launch, int *kinds) {
-    if (n < 0 || kl < 0 || ku < 0 || nrhs < 0) return -1;
-    return trfs_plan(n, kl, ku, nrhs, two_launch != 0, kinds);
+int bandlu_trfs_plan(int n, int kl, int ku, int nrhs, int batch, int phase, int *kinds) {
+    if (n < 0 || kl < 0 || ku < 0 || nrhs < 0 || batch < 0) return -1;
+    if ((phase & TRFS_TWO_LAUNCH) && (phase & TRFS_FUSED)) return -1;
+    return trfs_plan(n, kl, ku, nrhs, batch, phase, kinds);
 }
 
 int dgbtrf_strided_batched_ex(int m, int n, int kl, int ku, double *dA, int ldab, int64_t strideA, int *dipiv,
@@ -792,7 +869,8 @@ int dgbtrfs_strided_batched_ex(int n, int kl, int ku, int nrhs, double *dA, int 
         if (strideB < (int64_t)ldb * nrhs) return -12;
         if (!dinfo) return -13;
     }
-    if ((phase & ~TRFS_TWO_LAUNCH) < 0 || (phase & ~TRFS_TWO_LAUNCH) > 2) return -16;
+    if ((phase & TRFS_TWO_LAUNCH) && (phase & TRFS_FUSED)) return -16;
+    if ((phase & ~(TRFS_TWO_LAUNCH | TRFS_FUSED)) < 0 || (phase & ~(TRFS_TWO_LAUNCH | TRFS_FUSED)) > 2) return -16;
     return run_trfs(n, kl, ku, nrhs, Strided<double>{dA, strideA}, ldab, Strided<int>{dipiv, strideP},
                     Strided<double>{dB, strideB}, ldb, dinfo, batch, (cudaStream_t)stream, phase);
 }

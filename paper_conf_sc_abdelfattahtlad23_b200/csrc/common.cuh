@@ -121,6 +121,27 @@ __device__ __forceinline__ double ld_volatile_shared_f64(uint32_t a) {
     return v;
 }
 
+// Predicated global accesses (one instruction under a predicate, no branch).
+__device__ __forceinline__ void st_global_f64_if(bool p, double *a, double v) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %0, 0;\n\t@q st.global.f64 [%1], %2;\n\t}\n" ::"r"((int)p),
+                 "l"(a), "d"(v)
+                 : "memory");
+}
+__device__ __forceinline__ void ld_global_f64_if(bool p, const double *a, double &v) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %1, 0;\n\t@q ld.global.f64 %0, [%2];\n\t}\n"
+                 : "+d"(v)
+                 : "r"((int)p), "l"(a)
+                 : "memory");
+}
+
+// y = fma(a, b, y) (round to nearest) on lanes where p holds: one predicated DFMA
+// instead of an FMA and a 64-bit select.
+__device__ __forceinline__ void fma_rn_if(bool p, double a, double b, double &y) {
+    asm("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %1, 0;\n\t@q fma.rn.f64 %0, %2, %3, %0;\n\t}\n"
+        : "+d"(y)
+        : "r"((int)p), "d"(a), "d"(b));
+}
+
 // ---- mbarrier + bulk (TMA 1D) copies
 __device__ __forceinline__ void mbar_init(uint32_t bar, unsigned count) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(bar), "r"(count) : "memory");
@@ -162,6 +183,16 @@ __device__ __forceinline__ double ddiv_rn_if(bool p, double a, double b) {
     asm("mov.b64 %0, %1;" : "=d"(nb) : "d"(p ? b : 1.0));
     const double q = __ddiv_rn(na, nb);
     return p ? q : a;
+}
+
+// RN(1/x) for x != 0 and 0 for x == 0, without ever entering the slow path for
+// x == 0 (the operand passes an opaque move, as in ddiv_rn_if).  A zero result
+// marks a zero pivot (a finite nonzero x never has a zero reciprocal).
+__device__ __forceinline__ double drcp_rn_nz(double x) {
+    double xg;
+    asm("mov.b64 %0, %1;" : "=d"(xg) : "d"(x != 0.0 ? x : 1.0));
+    const double r = __drcp_rn(xg);
+    return x != 0.0 ? r : 0.0;
 }
 
 __host__ __device__ constexpr int pow2_ceil(int x) {

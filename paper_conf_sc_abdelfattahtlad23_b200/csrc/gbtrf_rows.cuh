@@ -337,6 +337,25 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
             const int pb = ps.pb, rb = ps.rb;
             const unsigned gb = ps.gb;
             const bool is_piv = (t == __ffs(gb) - 1);
+#ifdef BANDLU_ROWS_FASTCHAIN
+            // ---- (experiment, -DBANDLU_ROWS_FASTCHAIN) the step's dependency chain bypasses
+            // the shared-memory record: every lane computes RN(1/x) of its own candidate
+            // while the search runs, and the pivot lane's reciprocal, logical row and
+            // column-(j+1) entry -- all the next pivot search depends on -- arrive by shuffle.
+            // At 1,250 matrices per GPU the record write -> read -> RN(1/p) path held 15% of
+            // the stall samples, yet removing it measured 0.2341 vs 0.2343 ms (and 0.968 vs
+            // 0.960 ms at 10,000): the step time is its instruction count, not that chain.
+            const int plane = (int)gbase + max(__ffs(gb) - 1, 0);
+            double xs = x[0], u1s = VS(0, s + 1);
+#pragma unroll
+            for (int ri = 1; ri < R; ++ri) {
+                xs = (rb == ri) ? x[ri] : xs;
+                u1s = (rb == ri) ? VS(ri, s + 1) : u1s;
+            }
+            const double rinv = __shfl_sync(0xffffffffu, drcp_rn_nz(xs), plane);
+            const double u1 = __shfl_sync(0xffffffffu, u1s, plane);
+            const int ppos_f = __shfl_sync(0xffffffffu, pb, plane);
+#endif
 
             // ---- pivot row (U row j: slots s..s+KV) + (B entry, logical row) -> record s
             const uint32_t rcs = rec_s + (uint32_t)(s * WP * 8);
@@ -355,6 +374,10 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
 
             // ---- broadcast read (64-bit: one cycle per warp for all groups)
             const double2 yp = ld_shared_v2(rcs + RP * 8);
+#ifdef BANDLU_ROWS_FASTCHAIN
+            const int ppos = ppos_f;
+            const bool zp = (rinv == 0.0);
+#else
             const int ppos = (int)__double_as_longlong(yp.y);
 #ifdef BANDLU_ROWS_SHFL_P
             // pivot value straight from the pivot lane (off the record write -> read chain)
@@ -366,6 +389,7 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
             const double p = ld_volatile_shared_f64(rcs + s * 8);
 #endif
             const bool zp = (p == 0.0);
+#endif
 #ifndef BANDLU_ROWS_IPIV_STEP
             pv[s] = ppos + 1;  // stored once per block (C3 factorization 0.979 -> 0.960 ms)
 #else
@@ -382,7 +406,9 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
             }
 
             // ---- SCAL: multiplier = x * RN(1/p) (DSCAL(ONE/pivot), Q7)
+#ifndef BANDLU_ROWS_FASTCHAIN
             const double rinv = __drcp_rn(p);
+#endif
             double lu[R];
 #pragma unroll
             for (int ri = 0; ri < R; ++ri) {
@@ -416,10 +442,16 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
 #pragma unroll
             for (int h = (s + 1) / 2; h <= (s + KV) / 2; ++h) {
                 const double2 u2 = ld_shared_v2(rcs + h * 16);
+#ifdef BANDLU_ROWS_FASTCHAIN
+                // column j+1 (slot s+1) uses the shuffled value (bitwise the record's)
+                const double ua = (2 * h == s + 1) ? u1 : u2.x, ub = (2 * h + 1 == s + 1) ? u1 : u2.y;
+#else
+                const double ua = u2.x, ub = u2.y;
+#endif
 #pragma unroll
                 for (int ri = 0; ri < R; ++ri) {
-                    if (2 * h >= s + 1) VS(ri, 2 * h) = __fma_rn(lu[ri], -u2.x, VS(ri, 2 * h));
-                    if (2 * h + 1 <= s + KV) VS(ri, 2 * h + 1) = __fma_rn(lu[ri], -u2.y, VS(ri, 2 * h + 1));
+                    if (2 * h >= s + 1) VS(ri, 2 * h) = __fma_rn(lu[ri], -ua, VS(ri, 2 * h));
+                    if (2 * h + 1 <= s + KV) VS(ri, 2 * h + 1) = __fma_rn(lu[ri], -ub, VS(ri, 2 * h + 1));
                 }
                 // column j+1 (slot s+1) is final for step j+1: its pivot search overlaps the
                 // rest of this update

@@ -138,18 +138,23 @@ def test_product_package_does_not_import_oracle():
 
 def test_trfs_plan_reports_the_launches(lib):
     """bandlu_trfs_plan (no launch): the fused gbsv kernel for nrhs == 1 on row-slot
-    bands, forward-fused factorization + backward launch on other compiled bands,
-    trf + trs otherwise."""
+    bands while the batch fits in one wave of it, else the forward-fused factorization
+    + backward launch; trf + trs where no fused path exists."""
     from paper_conf_sc_abdelfattahtlad23_b200 import binding as b
-    p = b.trfs_plan(512, 10, 10, 1)
+    p = b.trfs_plan(512, 10, 10, 1, 1000)
     assert p == {"kernels": ["gbtrf_rows_kernel"], "bytes": ["gbsv"], "fused": True}
-    p = b.trfs_plan(512, 10, 10, 1, two_launch=True)
+    p = b.trfs_plan(512, 10, 10, 1, 10000)  # C3: 2.8 waves -> two launches
     assert p["kernels"] == ["gbtrf_rows_kernel", "gbtrs_bwd_kernel"] and p["bytes"] == ["trf_fwd", "trs_bwd"]
-    p = b.trfs_plan(2048, 32, 32, 1)
+    assert b.trfs_plan(512, 10, 10, 1, 10000, b.TRFS_FUSED)["fused"]
+    assert not b.trfs_plan(512, 10, 10, 1, 10, b.TRFS_TWO_LAUNCH)["fused"]
+    p = b.trfs_plan(2048, 32, 32, 1, 100)
     assert p["kernels"] == ["gbtrf_wide_kernel", "gbtrs_window_kernel"] and not p["fused"]
-    p = b.trfs_plan(1024, 2, 32, 16)
+    p = b.trfs_plan(1024, 2, 32, 1, 100)  # kl+ku+1+PF > 2G: no fused kernel for (2,32)
+    assert p["kernels"] == ["gbtrf_rows_kernel", "gbtrs_window_kernel"] and not p["fused"]
+    p = b.trfs_plan(1024, 2, 32, 16, 5000)
     assert p["kernels"] == ["gbtrf_rows_kernel", "gbtrs_window_kernel"] and p["bytes"] == ["trf", "trs"]
-    p = b.trfs_plan(100, 5, 9, 1)
+    p = b.trfs_plan(100, 5, 9, 1, 10)
     assert p["kernels"] == ["gbtrf_generic_kernel", "gbtrs_generic_kernel"]
-    assert b.trfs_plan(0, 1, 1, 1)["kernels"] == []
-    assert lib.bandlu_trfs_plan(-1, 1, 1, 1, 0, None) < 0
+    assert b.trfs_plan(0, 1, 1, 1, 10)["kernels"] == []
+    assert lib.bandlu_trfs_plan(-1, 1, 1, 1, 1, 0, None) < 0
+    assert lib.bandlu_trfs_plan(8, 1, 1, 1, 1, b.TRFS_TWO_LAUNCH | b.TRFS_FUSED, None) < 0

@@ -36,11 +36,13 @@ def _gpu_trf(A_np, m, n, kl, ku, variant=bl.AUTO):
     return A.cpu().numpy(), ipiv.cpu().numpy()[:, :min(m, n)], info.cpu().numpy()
 
 
-def trf_variants(kl, ku):
+def trf_variants(kl, ku, square=True):
     """Forced factorization variants to cross-check: the safeguard, the row-owner
-    window, and the row-slot (ROWS) and tensor-core (DMMA) kernels where they are
-    compiled for (kl, ku)."""
+    window, and the row-slot (ROWS), thread-per-matrix (TPM, square only) and
+    tensor-core (DMMA) kernels where they are compiled for (kl, ku)."""
     v = [bl.WINDOW, bl.GENERIC] if (kl, ku) in WINDOW_BANDS else [bl.GENERIC]
+    if square and bl.tpm_available(kl, ku):
+        v.append(bl.TPM)
     if bl.rows_available(kl, ku):
         v.append(bl.ROWS)
     if bl.tc_available(kl, ku):
@@ -63,7 +65,7 @@ def _check_trf(m, n, kl, ku, batch, variant, ldab=None, first=0, A_in=None):
 
 
 @pytest.mark.parametrize("kl,ku", ALL_BANDS)
-@pytest.mark.parametrize("variant", [bl.WINDOW, bl.GENERIC, bl.ROWS, bl.TC, bl.THREAD])
+@pytest.mark.parametrize("variant", [bl.WINDOW, bl.GENERIC, bl.ROWS, bl.TC, bl.THREAD, bl.TPM])
 @pytest.mark.parametrize("n", [1, 2, 7, 37, 100])
 def test_trf_parity_small(kl, ku, variant, n):
     if variant not in trf_variants(kl, ku):
@@ -76,7 +78,7 @@ def test_trf_parity_small(kl, ku, variant, n):
 @pytest.mark.parametrize("mn", [(30, 20), (20, 30), (5, 40), (40, 5), (1, 9), (9, 1)])
 def test_trf_parity_rectangular(kl, ku, mn):
     m, n = mn
-    for variant in trf_variants(kl, ku):
+    for variant in trf_variants(kl, ku, square=False):
         _check_trf(m, n, kl, ku, batch=9, variant=variant)
 
 
@@ -423,12 +425,13 @@ def _sample_indices(batch, seed=7, per_warp=(2, 4, 8, 16, 32), extra=48):
 
 
 @pytest.mark.parametrize("batch,n,kl,ku", TRFS_FULL)
-def test_trfs_full_batch_sampled_parity(batch, n, kl, ku):
+@pytest.mark.parametrize("phase", [0, bl.TRFS_FUSED])  # the library's plan (as bench.py), and the fused kernel
+def test_trfs_full_batch_sampled_parity(batch, n, kl, ku, phase):
     A = torch.from_numpy(I.gen_band(n, n, kl, ku, count=batch)).cuda()
     B = torch.from_numpy(I.gen_rhs(n, 1, count=batch)).cuda()
     P = torch.zeros((batch, n), dtype=torch.int32, device="cuda")
     info = torch.full((batch,), -7, dtype=torch.int32, device="cuda")
-    bl.dgbtrfs_strided_batched(n, kl, ku, A, P, B, info)
+    bl.dgbtrfs_strided_batched(n, kl, ku, A, P, B, info, phase=phase)
     torch.cuda.synchronize()
     sample = _sample_indices(batch)
     assert len(sample) >= 64 or len(sample) == batch
@@ -454,7 +457,7 @@ def test_trfs_full_batch_sampled_parity(batch, n, kl, ku):
 # n).  y(0..n-1) lives in shared memory when it fits (dgbsv may then leave B
 # untouched where info > 0), else in B (large n: dgbtrfs only; dgbsv takes two
 # launches).  Both plans must equal the oracle bitwise.
-FUSED_BANDS = [(10, 10), (10, 7), (2, 32), (1, 1), (2, 2), (2, 3), (4, 4)]
+FUSED_BANDS = [(10, 10), (10, 7), (1, 1), (2, 2), (2, 3), (4, 4)]  # (2,32): kv+1+PF > 2G, no fused kernel
 
 
 def _trfs(A_np, B_np, n, kl, ku, phase=0):
@@ -470,16 +473,16 @@ def _trfs(A_np, B_np, n, kl, ku, phase=0):
 @pytest.mark.parametrize("kl,ku", FUSED_BANDS)
 @pytest.mark.parametrize("n", [3, 17, 130, 777, 1000])  # 777 / 1000: y beyond the shared-memory budget at (10,10)
 def test_fused_gbsv_kernel_vs_oracle_and_two_launch_plan(kl, ku, n):
-    plan = bl.trfs_plan(n, kl, ku, 1)
-    assert plan["fused"] and plan["kernels"] == ["gbtrf_rows_kernel"]
-    assert bl.trfs_plan(n, kl, ku, 1, two_launch=True)["kernels"][0] == "gbtrf_rows_kernel"
     batch = 19  # ragged: not a multiple of matrices per warp / CTA
+    plan = bl.trfs_plan(n, kl, ku, 1, batch)
+    assert plan["fused"] and plan["kernels"] == ["gbtrf_rows_kernel"]
+    assert bl.trfs_plan(n, kl, ku, 1, batch, bl.TRFS_TWO_LAUNCH)["kernels"][0] == "gbtrf_rows_kernel"
     A = I.gen_band(n, n, kl, ku, count=batch, first=n)
     B = I.gen_rhs(n, 1, ldb=n + 2, count=batch, first=n)
     Ao, Bo = A.copy(), B.copy()
     ipo, info_o = oracle.dgbtrf(Ao, n, n, kl, ku)
     oracle.dgbtrs(Ao, ipo, Bo, n, kl, ku)
-    for phase in (0, bl.TRFS_TWO_LAUNCH):
+    for phase in (0, bl.TRFS_TWO_LAUNCH, bl.TRFS_FUSED):
         Ag, Pg, Bg, Ig = _trfs(A.copy(), B.copy(), n, kl, ku, phase)
         assert np.array_equal(Ig, info_o)
         assert np.array_equal(Pg, ipo)
@@ -487,7 +490,7 @@ def test_fused_gbsv_kernel_vs_oracle_and_two_launch_plan(kl, ku, n):
         assert np.all(same_bits(Bg, Bo))  # incl. the NaN ldb padding rows
 
 
-@pytest.mark.parametrize("kl,ku", FUSED_BANDS)
+@pytest.mark.parametrize("kl,ku", FUSED_BANDS + [(2, 32)])
 @pytest.mark.parametrize("n", [40, 512, 1000])
 def test_fused_dgbsv_leaves_b_untouched_where_singular(kl, ku, n):
     """dgbsv through the fused kernel (y in shared memory; n = 1000 at (10,10)

@@ -16,8 +16,9 @@ from paper_conf_sc_abdelfattahtlad23_b200 import inputs as I  # noqa: E402
 cfg = sys.argv[1] if len(sys.argv) > 1 else "C3"
 reps = int(sys.argv[2]) if len(sys.argv) > 2 else 1
 bpg, n, kl, ku, nrhs, _ = bench.CONFIGS[cfg]
-A0 = torch.from_numpy(I.gen_band(n, n, kl, ku, count=bpg)).cuda()
-B0 = torch.from_numpy(I.gen_rhs(n, nrhs, count=bpg)).cuda()
+bpg = int(os.environ.get("PROF_BATCH", bpg))
+A0 = I.gen_band_torch(n, n, kl, ku, count=bpg, device='cuda')
+B0 = I.gen_rhs_torch(n, nrhs, count=bpg, device='cuda')
 A, B = torch.empty_like(A0), torch.empty_like(B0)
 P = torch.zeros((bpg, n), dtype=torch.int32, device="cuda")
 info = torch.zeros(bpg, dtype=torch.int32, device="cuda")
@@ -27,8 +28,8 @@ for _ in range(reps):
     if os.environ.get("PROF_SEPARATE"):  # plain dgbtrf + dgbtrs launches
         bl.dgbtrf_strided_batched(n, n, kl, ku, A, P, info)
         bl.dgbtrs_strided_batched("N", n, kl, ku, A, P, B)
-    else:  # the bench step: dgbtrfs (fused forward solve when nrhs == 1), two launches
-        bl.dgbtrfs_strided_batched(n, kl, ku, A, P, B, info, phase=1)
-        bl.dgbtrfs_strided_batched(n, kl, ku, A, P, B, info, phase=2)
+    else:  # the bench step: dgbtrfs, every launch of its plan (PROF_TWO: the two-launch plan)
+        x = bl.TRFS_TWO_LAUNCH if os.environ.get("PROF_TWO") else 0
+        bl.dgbtrfs_strided_batched(n, kl, ku, A, P, B, info, phase=x)
 torch.cuda.synchronize()
 print("ok", cfg, int(info.abs().sum()))
