@@ -216,6 +216,18 @@ int bandlu_rows_available(int kl, int ku);
 int bandlu_thread_available(int kl, int ku);
 /* 1 if a thread-per-matrix shared-memory-window kernel (BANDLU_TPM) is compiled for (kl, ku), else 0. */
 int bandlu_tpm_available(int kl, int ku);
+/* Run-time compiled bands (Sec. 8.1: JIT-compiled register-resident
+ * kernels).  A (kl, ku) that no ahead-of-time instantiation covers takes the same kernel
+ * templates compiled with NVRTC for sm_100a on the first call that needs them (seconds;
+ * cached per process, and on disk when BANDLU_JIT_CACHE names a directory): the row-slot
+ * factorization for kl <= 27, the two-warp one for kl <= 59, the backward / window
+ * solves; strided entry points only (pointer arrays use the generic kernels).  Without
+ * NVRTC (dlopen libnvrtc.so.12) or with BANDLU_JIT=0 such bands use the generic kernels.
+ * bandlu_jit_band: 1 if (kl, ku) is served that way (no compilation).  bandlu_jit_check:
+ * compile (no GPU needed, nothing loaded) every kernel the band uses; 0 on success, else 1
+ * and the first compiler error in log (loglen bytes). */
+int bandlu_jit_band(int kl, int ku);
+int bandlu_jit_check(int kl, int ku, char *log, int loglen);
 /* 1 if a lane-per-row solve kernel (dgbtrs BANDLU_ROWS) is compiled for (kl, ku), else 0. */
 int bandlu_trs_rows_available(int kl, int ku);
 /* The launches one dgbtrfs_strided_batched call with this phase flag set makes

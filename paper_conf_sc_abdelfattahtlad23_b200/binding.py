@@ -72,6 +72,8 @@ def load(build_if_missing: bool = False):
         "bandlu_trs_rows_available": [i, i],
         "bandlu_thread_available": [i, i],
         "bandlu_tpm_available": [i, i],
+        "bandlu_jit_band": [i, i],
+        "bandlu_jit_check": [i, i, p, i],
         "bandlu_trs_variant": [i, i, i, i],
         "bandlu_trfs_plan": [i, i, i, i, i, i, p],
         "bandlu_version": [],
@@ -88,7 +90,7 @@ def load(build_if_missing: bool = False):
 EXPORTS = ("dgbtrf_batched", "dgbtrf_strided_batched", "dgbtrf_strided_batched_ex", "dgbtrs_batched",
            "dgbtrs_strided_batched", "dgbtrs_strided_batched_ex", "dgbsv_batched", "dgbsv_strided_batched",
            "dgbsv_strided_batched_host", "dgbtrfs_strided_batched", "dgbtrfs_strided_batched_ex", "bandlu_trf_variant", "bandlu_trs_variant", "bandlu_tc_available", "bandlu_rows_available", "bandlu_trs_rows_available", "bandlu_thread_available",
-           "bandlu_tpm_available", "bandlu_trfs_plan", "bandlu_version")
+           "bandlu_tpm_available", "bandlu_jit_band", "bandlu_jit_check", "bandlu_trfs_plan", "bandlu_version")
 
 
 def _stream(stream):
@@ -248,6 +250,18 @@ def thread_available(kl: int, ku: int) -> bool:
 def tpm_available(kl: int, ku: int) -> bool:
     """True if the thread-per-matrix shared-memory-window factorization (variant TPM) is compiled for (kl, ku)."""
     return bool(load().bandlu_tpm_available(kl, ku))
+
+
+def jit_band(kl: int, ku: int) -> bool:
+    """True if (kl, ku) is served by run-time compiled (NVRTC) kernels (include/bandlu.h)."""
+    return bool(load().bandlu_jit_band(kl, ku))
+
+
+def jit_check(kl: int, ku: int) -> str:
+    """Compile (no GPU needed) every run-time kernel the band uses; "" on success, else the error."""
+    buf = ctypes.create_string_buffer(8192)
+    rc = load().bandlu_jit_check(kl, ku, buf, len(buf))
+    return "" if rc == 0 else buf.value.decode(errors="replace") or "failed"
 
 
 def trs_rows_available(kl: int, ku: int) -> bool:

@@ -24,6 +24,7 @@
 #include "gbtrs_rows.cuh"
 #include "gbtrs_window.cuh"
 #include "generic.cuh"
+#include "jit.cuh"
 
 using namespace bandlu;
 
@@ -310,8 +311,85 @@ bool trf_tc_available(int kl, int ku) {
     return false;
 }
 
+// ---- run-time compiled bands (jit.cuh): any (kl, ku) that no list above instantiates
+// takes the row-slot kernel (kl + 5 <= 32 lanes: G = pow2 >= kl + 5) or the two-warp
+// wide kernel (kl + 5 <= 64), compiled on first use; strided entry points only.
+bool trf_compiled(int kl, int ku) { return trf_rows_available(kl, ku) || trf_window_available(kl, ku); }
+int jit_rows_g(int kl) {
+    int g = 8;
+    while (g < kl + 5) g *= 2;
+    return g <= 32 ? g : 0;
+}
+bool jit_band(int kl, int ku) {
+    return !trf_compiled(kl, ku) && (jit_rows_g(kl) > 0 || kl + 5 <= 64) && bandlu_jit::nvrtc().ok;
+}
+const bandlu_jit::Kern &jit_trf(int kl, int ku, int fl) {
+    const int g = jit_rows_g(kl);
+    return g ? bandlu_jit::rows(kl, ku, g, fl) : bandlu_jit::wide(kl, ku, (fl & FL_FWD) != 0);
+}
+int jit_launch_trf(const bandlu_jit::Kern &K, int kl, int fl, int m, int n, Strided<double> A, int ldab,
+                   Strided<int> P, int *info, int batch, cudaStream_t st, Strided<double> B) {
+    void *args[] = {&m, &n, &A, &ldab, &P, &info, &batch, &B};
+    if (jit_rows_g(kl)) {
+        const long long W = K.geo[0], GPW = K.geo[1], GD = K.geo[3];
+        const size_t sm = (size_t)(W * GPW * (GD + ((fl & FL_YSM) ? ((n + 15) & ~15) : 0)) * 8);
+        if (sm > 48 * 1024) {
+            cudaError_t e = cudaFuncSetAttribute((const void *)K.k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+            if (e != cudaSuccess) return cuda_ret(e);
+        }
+        const unsigned grid = (unsigned)((batch + W * GPW - 1) / (W * GPW));
+        return cuda_ret(cudaLaunchKernel((const void *)K.k, dim3(grid), dim3((unsigned)(W * 32)), args, sm, st));
+    }
+    const size_t sm = (size_t)K.geo[0];
+    if (sm > 48 * 1024) {
+        cudaError_t e = cudaFuncSetAttribute((const void *)K.k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+        if (e != cudaSuccess) return cuda_ret(e);
+    }
+    return cuda_ret(cudaLaunchKernel((const void *)K.k, dim3((unsigned)batch), dim3(64), args, sm, st));
+}
+// run-time compiled window solve (any nrhs); skip: info array (dgbsv) or nullptr; fwd 0: backward only
+int jit_launch_trs_window(int kl, int ku, int n, int nrhs, Strided<const double> A, int ldab, Strided<const int> P,
+                          Strided<double> B, int ldb, const int *skip, int batch, cudaStream_t st, int fwd) {
+    int R = nrhs >= 32 ? 32 : pow2_ceil(nrhs);
+    int chunks = (nrhs + 31) / 32;
+    const bool pairs = R >= 2;
+    const bandlu_jit::Kern &K = bandlu_jit::window(kl, ku, pairs);
+    if (!K.ok) return BANDLU_ERR_UNSUPPORTED;
+    const int64_t units = (int64_t)batch * chunks;
+    int gpw = 32 / R;
+    while (gpw > 1 && units < (int64_t)gpw * kTrsWarpsTarget) gpw >>= 1;
+    int li = 0;
+    while ((1 << li) < R) ++li;
+    const size_t sm = (size_t)(K.geo[0] + (long long)gpw * K.geo[1 + li]) * 8;
+    if (sm > 48 * 1024) {
+        cudaError_t e = cudaFuncSetAttribute((const void *)K.k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+        if (e != cudaSuccess) return cuda_ret(e);
+    }
+    const unsigned grid = (unsigned)((units + gpw - 1) / gpw);
+    void *args[] = {&n, &nrhs, &A, &ldab, &P, &B, &ldb, &skip, &batch, &R, &chunks, &gpw, &fwd};
+    return cuda_ret(cudaLaunchKernel((const void *)K.k, dim3(grid), dim3(32), args, sm, st));
+}
+// run-time compiled backward-only solve (kl + ku + 1 <= 32), matrices per warp as launch_trs_bwd_lean
+int jit_launch_trs_bwd(int kl, int ku, int n, Strided<const double> A, int ldab, Strided<double> B, int batch,
+                       cudaStream_t st) {
+    int gpw = 32;
+    while (gpw > 1 && batch < (int64_t)gpw * kTrsWarpsTarget) gpw >>= 1;
+    gpw = gpw < 2 ? 2 : gpw;
+    const bandlu_jit::Kern &K = bandlu_jit::bwd(kl, ku, gpw);
+    if (!K.ok) return BANDLU_ERR_UNSUPPORTED;
+    const size_t sm = (size_t)(K.geo[0] + K.geo[1] * gpw) * 8;
+    if (sm > 48 * 1024) {
+        cudaError_t e = cudaFuncSetAttribute((const void *)K.k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+        if (e != cudaSuccess) return cuda_ret(e);
+    }
+    const unsigned grid = (unsigned)((batch + gpw - 1) / gpw);
+    void *args[] = {&n, &A, &ldab, &B, &batch};
+    return cuda_ret(cudaLaunchKernel((const void *)K.k, dim3(grid), dim3(32), args, sm, st));
+}
+
 int pick_trf(int m, int n, int kl, int ku) {
     if (m <= 0 || n <= 0) return BANDLU_GENERIC;
+    if (jit_band(kl, ku)) return BANDLU_ROWS;  // compiled on first use (jit.cuh)
     // BANDLU_TC is opt-in: measured slower than the row-owner window at C3
     // (1.54 vs 1.10 ms), so AUTO never picks it.
     if (trf_thread_preferred(kl, ku)) return BANDLU_THREAD;
@@ -365,6 +443,15 @@ int run_trf(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int b
     if (kl == a && ku == b) return launch_trf_wide<a, b, false>(m, n, A, ldab, P, info, batch, st, Strided<double>{nullptr, 0});
         BANDLU_WIDE_LIST(X)
 #undef X
+        if constexpr (std::is_same_v<AP, Strided<double>>) {
+            if (jit_band(kl, ku)) {
+                const bandlu_jit::Kern &K = jit_trf(kl, ku, 0);
+                if (K.ok) return jit_launch_trf(K, kl, 0, m, n, A, ldab, P, info, batch, st, Strided<double>{nullptr, 0});
+            }
+            if (jit_band(kl, ku)) return launch_trf_generic(m, n, kl, ku, A, ldab, P, info, batch, st);
+        } else {
+            if (jit_band(kl, ku)) return launch_trf_generic(m, n, kl, ku, A, ldab, P, info, batch, st);
+        }
         return BANDLU_ERR_UNSUPPORTED;
     }
     if (variant == BANDLU_WINDOW && m > 0 && n > 0) {
@@ -431,10 +518,15 @@ bool trs_rows_preferred(int, int) { return false; }
 bool trs_rows_preferred(int kl, int ku) { return kl + ku + 1 <= 4 && trs_rows_available(kl, ku); }
 #endif
 
+// run-time compiled window solve for bands without a compiled one (jit.cuh)
+bool jit_trs_band(int kl, int ku) {
+    return !trs_window_available(kl, ku) && kl + ku <= 64 && bandlu_jit::nvrtc().ok;
+}
+
 int pick_trs(int n, int kl, int ku, int nrhs) {
     (void)n;
     if (nrhs == 1 && trs_rows_preferred(kl, ku)) return BANDLU_ROWS;
-    return trs_window_available(kl, ku) ? BANDLU_WINDOW : BANDLU_GENERIC;
+    return (trs_window_available(kl, ku) || jit_trs_band(kl, ku)) ? BANDLU_WINDOW : BANDLU_GENERIC;
 }
 
 template <class AP, class PP, class BP>
@@ -460,6 +552,13 @@ int run_trs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ldb
     if (kl == a && ku == b) return launch_trs_window<a, b>(n, nrhs, A, ldab, P, B, ldb, skip, batch, st);
         BANDLU_TRS_LIST(X)
 #undef X
+        if (jit_trs_band(kl, ku)) {
+            if constexpr (std::is_same_v<AP, Strided<const double>>) {
+                const int r = jit_launch_trs_window(kl, ku, n, nrhs, A, ldab, P, B, ldb, skip, batch, st, 1);
+                if (r != BANDLU_ERR_UNSUPPORTED) return r;
+            }
+            return launch_trs_generic(n, kl, ku, nrhs, A, ldab, P, B, ldb, skip, batch, st);
+        }
         return BANDLU_ERR_UNSUPPORTED;
     }
     if (variant == BANDLU_ROWS) {
@@ -584,11 +683,34 @@ enum { KN_TRF_ROWS = 1, KN_TRF_WINDOW, KN_TRF_WIDE, KN_TRF_THREAD, KN_TRF_GENERI
        KN_TRS_WINDOW, KN_TRS_GENERIC };
 enum { KB_TRF = 1, KB_TRF_FWD, KB_TRS_BWD, KB_TRS, KB_GBSV };
 
+// run-time compiled bands, nrhs == 1: is the fused kernel picked?  (geometry from the
+// compiled module: [0] WARPS, [1] GPW, [2] MINB, [3] GROUP_DBL, [4] fused solve ok)
+bool jit_fused_pick(const bandlu_jit::Kern &K, int kl, int64_t batch, int phase) {
+    if (!K.ok || !jit_rows_g(kl) || !K.geo[4] || (phase & TRFS_TWO_LAUNCH)) return false;
+    return (phase & TRFS_FUSED) || batch <= (int64_t)sm_count() * K.geo[2] * K.geo[0] * K.geo[1];
+}
+bool jit_ysm_fits(const bandlu_jit::Kern &K, int n) {
+    const size_t b = (size_t)(K.geo[0] * K.geo[1] * (K.geo[3] + ((n + 15) & ~15)) * 8);
+    return b <= kSmemPerSM && b * (size_t)K.geo[2] <= kSmemPerSM;
+}
+
 // the launches one dgbtrfs call makes for the shape (what run_trfs does)
 int trfs_plan(int n, int kl, int ku, int nrhs, int64_t batch, int phase, int *kinds) {
     int k = 0;
     auto put = [&](int name, int bytes) { if (kinds) kinds[k] = name * 16 + bytes; ++k; };
     if (n <= 0 || nrhs <= 0) return 0;
+    if (nrhs == 1 && jit_band(kl, ku)) {
+        const bandlu_jit::Kern &K = jit_trf(kl, ku, FL_FWD);
+        if (K.ok) {
+            if (jit_fused_pick(K, kl, batch, phase)) {
+                put(KN_TRF_ROWS, KB_GBSV);
+                return k;
+            }
+            put(jit_rows_g(kl) ? KN_TRF_ROWS : KN_TRF_WIDE, KB_TRF_FWD);
+            put(kl + ku + 1 <= 32 ? KN_TRS_BWD : KN_TRS_WINDOW, KB_TRS_BWD);
+            return k;
+        }
+    }
     if (trfs_fused_pick(n, kl, ku, nrhs, batch, phase)) {
         put(KN_TRF_ROWS, KB_GBSV);
         return k;
@@ -614,6 +736,7 @@ template <class AP, class PP, class BP>
 int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ldb, int *info, int batch,
              cudaStream_t st, int phase) {
     const bool fused = trfs_fused_pick(n, kl, ku, nrhs, batch, phase);
+    const int pflags = phase & (TRFS_TWO_LAUNCH | TRFS_FUSED);
     phase &= ~(TRFS_TWO_LAUNCH | TRFS_FUSED);
     if (batch == 0) return 0;
     if (fused) {
@@ -673,6 +796,29 @@ int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ld
 #undef X
         return r;
     }
+    if (n > 0 && nrhs == 1 && jit_band(kl, ku)) {  // run-time compiled band (jit.cuh)
+        const bandlu_jit::Kern &K = jit_trf(kl, ku, FL_FWD);
+        if (K.ok) {
+            const int ph = phase;
+            if (jit_fused_pick(K, kl, batch, pflags)) {
+                if (ph == 2) return 0;
+                const int fl = FL_FWD | FL_BWD | (jit_ysm_fits(K, n) ? FL_YSM : 0);
+                const bandlu_jit::Kern &KF = jit_trf(kl, ku, fl);
+                if (KF.ok) return jit_launch_trf(KF, kl, fl, n, n, A, ldab, P, info, batch, st, B);
+            } else {
+                int r = 0;
+                if (ph != 2) r = jit_launch_trf(K, kl, FL_FWD, n, n, A, ldab, P, info, batch, st, B);
+                if (r == 0 && ph != 1) {
+                    Strided<const double> Ac{A.base, A.stride};
+                    Strided<const int> Pc{P.base, P.stride};
+                    r = (kl + ku + 1 <= 32) ? jit_launch_trs_bwd(kl, ku, n, Ac, ldab, B, batch, st)
+                                            : jit_launch_trs_window(kl, ku, n, 1, Ac, ldab, Pc, B, ldb, nullptr, batch,
+                                                                    st, 0);
+                }
+                return r;
+            }
+        }
+    }
     if (phase != 2)
         if (int r = run_trf(n, n, kl, ku, A, ldab, P, info, batch, st, BANDLU_AUTO)) return r;
     if (phase == 1) return 0;
@@ -695,6 +841,14 @@ int run_gbsv(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ld
     }
         BANDLU_ROWS_LIST(X)
 #undef X
+    }
+    if (n > 0 && nrhs == 1 && jit_band(kl, ku)) {  // run-time compiled band: the fused kernel (jit.cuh)
+        const bandlu_jit::Kern &K = jit_trf(kl, ku, FL_FWD);
+        if (K.ok && jit_fused_pick(K, kl, batch, 0) && jit_ysm_fits(K, n)) {
+            const int fl = FL_FWD | FL_BWD | FL_YSM | FL_SKIPI;
+            const bandlu_jit::Kern &KF = jit_trf(kl, ku, fl);
+            if (KF.ok) return jit_launch_trf(KF, kl, fl, n, n, A, ldab, P, info, batch, st, B);
+        }
     }
     if (int r = run_trf(n, n, kl, ku, A, ldab, P, info, batch, st, BANDLU_AUTO)) return r;
     return run_trs(n, kl, ku, nrhs, Strided<const double>{A.base, A.stride}, ldab,
@@ -772,6 +926,40 @@ int bandlu_tc_available(int kl, int ku) { return trf_tc_available(kl, ku) ? 1 : 
 int bandlu_rows_available(int kl, int ku) { return trf_rows_available(kl, ku) ? 1 : 0; }
 int bandlu_thread_available(int kl, int ku) { return trf_thread_available(kl, ku) ? 1 : 0; }
 int bandlu_tpm_available(int kl, int ku) { return trf_tpm_available(kl, ku) ? 1 : 0; }
+
+// 1 if (kl, ku) is served by run-time compiled kernels (jit.cuh), else 0 (no compilation)
+int bandlu_jit_band(int kl, int ku) { return jit_band(kl, ku) ? 1 : 0; }
+
+// NVRTC-compile (no load, no GPU needed) the kernels a run-time compiled band uses: the
+// factorization (plain, + forward, fused) and the solves.  0 = every kernel compiled;
+// otherwise 1 and the first error in log (truncated to loglen).
+int bandlu_jit_check(int kl, int ku, char *log, int loglen) {
+    std::vector<bandlu_jit::Spec> specs;
+    const int g = jit_rows_g(kl);
+    if (g) {
+        specs.push_back(bandlu_jit::rows_spec(kl, ku, g, 0));
+        specs.push_back(bandlu_jit::rows_spec(kl, ku, g, FL_FWD));
+        if (kl + ku + 1 + BANDLU_FUSED_PF <= 2 * g)  // FusedSolve<kv, g>::ok
+            specs.push_back(bandlu_jit::rows_spec(kl, ku, g, FL_FWD | FL_BWD | FL_YSM));
+    } else {
+        specs.push_back(bandlu_jit::wide_spec(kl, ku, true));
+    }
+    if (kl + ku + 1 <= 32) specs.push_back(bandlu_jit::bwd_spec(kl, ku, 8));
+    specs.push_back(bandlu_jit::window_spec(kl, ku, true));
+    for (const auto &sp : specs) {
+        std::vector<char> bin;
+        std::string low;
+        const std::string err = bandlu_jit::compile(sp.first, sp.second, bin, low);
+        if (!err.empty()) {
+            if (log && loglen > 0) {
+                std::strncpy(log, err.c_str(), (size_t)loglen - 1);
+                log[loglen - 1] = '\0';
+            }
+            return 1;
+        }
+    }
+    return 0;
+}
 int bandlu_trs_rows_available(int kl, int ku) { return trs_rows_available(kl, ku) ? 1 : 0; }
 int bandlu_trs_variant(int n, int kl, int ku, int nrhs) { return pick_trs(n, kl, ku, nrhs); }
 int bandlu_trfs_plan(int n, int kl, int ku, int nrhs, int batch, int phase, int *kinds) {

@@ -1,8 +1,23 @@
 // common.cuh -- batch addressing and small PTX helpers shared by the sm_100a
 // band LU / solve kernels.  (No arithmetic of the method lives here.)
 #pragma once
+#ifdef __CUDACC_RTC__
+// run-time compilation (jit.cuh, NVRTC): no host headers; the few types used here
+typedef unsigned int uint32_t;
+typedef unsigned long long uint64_t;
+typedef long long int64_t;
+typedef unsigned long long uintptr_t;
+typedef unsigned long size_t;
+namespace std {
+template <class T, T v>
+struct integral_constant {
+    static constexpr T value = v;
+};
+}  // namespace std
+#else
 #include <cstdint>
 #include <cuda_runtime.h>
+#endif
 
 namespace bandlu {
 

@@ -34,12 +34,17 @@ struct TrfWide {
     static constexpr int RP = WP - 2;
     static constexpr int D = 4, DB = D / U;
     static constexpr int RR = pow2_ceil((DB + 1) * U);
+#ifdef BANDLU_WIDE_ONESYNC
+    static constexpr int NREC = 2 * U;  // one candidate record per warp and step (one barrier per step)
+#else
     static constexpr int NREC = U;
+#endif
     static constexpr int BK = W + U - 1;
     static constexpr int BIT = (BK * U + G - 1) / G;
     static_assert(BIT <= 32, "block element mask");
-    // ring + records + per-warp argmax exchange (2 x 16 B) + per-warp free-slot counts (16 B)
-    static constexpr size_t smem_bytes() { return (size_t)((RR + NREC) * WP + 6) * sizeof(double); }
+    // ring + records + per-warp argmax exchange (2 x 2 x 16 B, double-buffered by step parity)
+    // + per-warp free-slot counts (16 B)
+    __host__ __device__ static constexpr size_t smem_bytes() { return (size_t)((RR + NREC) * WP + 10) * sizeof(double); }
 };
 
 template <int KL, int KU, bool FWD, class AP, class PP, class BP>
@@ -65,7 +70,7 @@ __global__ void __launch_bounds__(64, 4)
     const uint32_t ring_s = smem_u32(ring);
     const uint32_t rec_s = ring_s + RR * WP * 8;
     uint4 *xch = reinterpret_cast<uint4 *>(smem + (RR + C::NREC) * WP);  // [2]: (hi, lo, pos, valid)
-    unsigned *fcnt = reinterpret_cast<unsigned *>(xch + 2);               // [2]: free slots per warp
+    unsigned *fcnt = reinterpret_cast<unsigned *>(xch + 4);               // [2]: free slots per warp
 
     for (int i = t; i < RR * WP; i += G) ring[i] = 0.0;
     __syncthreads();
@@ -123,8 +128,12 @@ __global__ void __launch_bounds__(64, 4)
     double *colj = ab + KV;
     double *colb = ab;
     int pv[U];  // the block's pivots (1-based), stored once per block by thread 0 (as gbtrf_rows.cuh)
+    int wsel[U];  // which warp's record holds step s's pivot row
 #pragma unroll
-    for (int s = 0; s < U; ++s) pv[s] = 0;
+    for (int s = 0; s < U; ++s) {
+        pv[s] = 0;
+        wsel[s] = 0;
+    }
     const unsigned below = (1u << lane) - 1u;
 #pragma unroll 1
     for (int j0 = 0; j0 < mn; j0 += U) {
@@ -165,6 +174,26 @@ __global__ void __launch_bounds__(64, 4)
                 gb = __ballot_sync(0xffffffffu, cand && (unsigned)pos == pp);
             }
             const int wl = __ffs(gb) - 1;  // this warp's best lane (-1: no candidate)
+#ifdef BANDLU_WIDE_ONESYNC
+            // ---- each warp's best candidate row -> its record (s, w); ONE barrier, then every
+            // lane picks the winner (warp 1 wins on a larger key, or an equal key with the
+            // smaller logical row) and reads the winner's record
+            const bool wbest = (lane == wl);
+            if (lane == (wl < 0 ? 0 : wl))
+                xch[(s & 1) * 2 + w] = make_uint4(kh, kl, (unsigned)pos, wl < 0 ? 0u : 1u);
+            {
+                const uint32_t rcw = rec_s + (uint32_t)((2 * s + w) * WP * 8);
+#pragma unroll
+                for (int h = s / 2; h <= (s + KV) / 2; ++h) st_shared_v2_if(wbest, rcw + h * 16, v[h]);
+                st_shared_v2_if(wbest, rcw + RP * 8, make_double2(bq, __longlong_as_double((long long)pos)));
+            }
+            __syncthreads();
+            const uint4 c0 = xch[(s & 1) * 2], c1 = xch[(s & 1) * 2 + 1];
+            const bool w1 = c1.w && (!c0.w || c1.x > c0.x || (c1.x == c0.x && (c1.y > c0.y || (c1.y == c0.y && c1.z < c0.z))));
+            const bool is_piv = (w == (w1 ? 1 : 0)) && wbest;
+            const uint32_t rcs = rec_s + (uint32_t)((2 * s + (w1 ? 1 : 0)) * WP * 8);
+            wsel[s] = w1 ? 1 : 0;
+#else
             if (lane == (wl < 0 ? 0 : wl))
                 xch[w] = make_uint4(kh, kl, (unsigned)pos, wl < 0 ? 0u : 1u);
             __syncthreads();
@@ -179,6 +208,7 @@ __global__ void __launch_bounds__(64, 4)
             for (int h = s / 2; h <= (s + KV) / 2; ++h) st_shared_v2_if(is_piv, rcs + h * 16, v[h]);
             st_shared_v2_if(is_piv, rcs + RP * 8, make_double2(bq, __longlong_as_double((long long)pos)));
             __syncthreads();
+#endif
             const double2 yp = ld_shared_v2(rcs + RP * 8);
             const int ppos = (int)__double_as_longlong(yp.y);
             const double p = ld_volatile_shared_f64(rcs + s * 8);
@@ -219,8 +249,16 @@ __global__ void __launch_bounds__(64, 4)
 #pragma unroll
         for (int k = 0; k < BIT; ++k) {
             const int e = t + k * G, bs = e % U, bk = e / U;
+#ifdef BANDLU_WIDE_ONESYNC
+            int ws = wsel[0];
+#pragma unroll
+            for (int q = 1; q < U; ++q) ws = (bs == q) ? wsel[q] : ws;
+            if ((bmask >> k & 1u) && j0 + bs < mn && j0 + bk < n)
+                colb[boff(k) + KV] = ld_shared_f64(rec_s + (uint32_t)(((2 * bs + ws) * WP + bk) * 8));
+#else
             if ((bmask >> k & 1u) && j0 + bs < mn && j0 + bk < n)
                 colb[boff(k) + KV] = ld_shared_f64(rec_s + (uint32_t)((bs * WP + bk) * 8));
+#endif
         }
         colb += (int64_t)U * ldab;
         if (t == 0) {

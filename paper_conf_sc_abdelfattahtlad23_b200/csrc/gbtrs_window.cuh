@@ -36,7 +36,9 @@
 #pragma once
 #include "common.cuh"
 
+#ifndef __CUDACC_RTC__
 #include <type_traits>
+#endif
 
 #ifndef BANDLU_TRS_NS_NARROW
 #define BANDLU_TRS_NS_NARROW 16

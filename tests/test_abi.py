@@ -115,7 +115,8 @@ def test_variant_heuristic_is_shape_only(lib):
     assert b.trf_variant(256, 256, 1, 1) == b.ROWS  # thin bands: row-slot kernel too
     assert b.trf_variant(64, 64, 0, 3) == b.WINDOW
     assert b.trf_variant(100, 100, 32, 32) == b.ROWS  # kl+1 > 32 lanes: two-warp row-slot kernel
-    assert b.trf_variant(100, 100, 33, 20) == b.GENERIC  # band not compiled: safeguard kernel
+    # band not instantiated ahead of time: run-time compiled row-slot kernels (NVRTC), else the safeguard
+    assert b.trf_variant(100, 100, 33, 20) == (b.ROWS if b.jit_band(33, 20) else b.GENERIC)
     assert b.trs_variant(100, 32, 32, 1) == b.WINDOW
     assert b.trf_variant(0, 5, 1, 1) == b.GENERIC
     assert b.trs_variant(1024, 2, 32, 16) == b.WINDOW
@@ -153,8 +154,24 @@ def test_trfs_plan_reports_the_launches(lib):
     assert p["kernels"] == ["gbtrf_rows_kernel", "gbtrs_window_kernel"] and not p["fused"]
     p = b.trfs_plan(1024, 2, 32, 16, 5000)
     assert p["kernels"] == ["gbtrf_rows_kernel", "gbtrs_window_kernel"] and p["bytes"] == ["trf", "trs"]
-    p = b.trfs_plan(100, 5, 9, 1, 10)
-    assert p["kernels"] == ["gbtrf_generic_kernel", "gbtrs_generic_kernel"]
+    p = b.trfs_plan(100, 5, 9, 1, 10, b.TRFS_TWO_LAUNCH)  # (5,9): not instantiated ahead of time
+    if b.jit_band(5, 9):  # run-time compiled (NVRTC) kernels
+        assert p["kernels"][0] == "gbtrf_rows_kernel" and p["kernels"][1] in ("gbtrs_bwd_kernel", "gbtrs_window_kernel")
+    else:
+        assert p["kernels"] == ["gbtrf_generic_kernel", "gbtrs_generic_kernel"]
     assert b.trfs_plan(0, 1, 1, 1, 10)["kernels"] == []
     assert lib.bandlu_trfs_plan(-1, 1, 1, 1, 1, 0, None) < 0
     assert lib.bandlu_trfs_plan(8, 1, 1, 1, 1, b.TRFS_TWO_LAUNCH | b.TRFS_FUSED, None) < 0
+
+
+def test_jit_bands_compile_without_gpu(lib):
+    """Every kernel a run-time compiled band uses compiles with NVRTC for sm_100a from
+    the sources embedded in the library (no GPU needed): row-slot bands (incl. fused
+    solve), a wide band (kl + 1 > 32) and a band without a fused solve (kv + 9 > 2G)."""
+    from paper_conf_sc_abdelfattahtlad23_b200 import binding as b
+    if not b.jit_band(5, 6):
+        pytest.skip("NVRTC not available")
+    for kl, ku in [(5, 6), (16, 16), (0, 40), (33, 20)]:
+        assert b.jit_band(kl, ku)
+        assert b.jit_check(kl, ku) == "", (kl, ku)
+    assert not b.jit_band(10, 10) and not b.jit_band(2, 32)  # instantiated ahead of time

@@ -517,3 +517,71 @@ def test_fused_dgbsv_leaves_b_untouched_where_singular(kl, ku, n):
     assert np.all(same_bits(Bgn, Bo))
     for b in (2, 5, 9):
         assert np.all(same_bits(Bgn[b], B[b]))
+
+
+# ------------------------------------------- run-time compiled bands (NVRTC)
+# Bands no list instantiates ahead of time run the same templates compiled with
+# NVRTC on first use (jit.cuh; Sec. 8.1): every entry point and
+# plan must still equal the oracle bitwise.
+JIT_BANDS = [(5, 6), (16, 16), (20, 20), (0, 32), (7, 1), (33, 20)]
+
+
+@pytest.mark.parametrize("kl,ku", JIT_BANDS)
+def test_jit_band_parity(kl, ku):
+    if not bl.jit_band(kl, ku):
+        pytest.skip("NVRTC not available")
+    n, batch = 150, 37
+    A0 = I.gen_band(n, n, kl, ku, count=batch, first=kl * 100 + ku)
+    B0 = I.gen_rhs(n, 3, ldb=n + 1, count=batch)
+    Ao = A0.copy()
+    ipo, info_o = oracle.dgbtrf(Ao, n, n, kl, ku)
+    Bo = B0.copy()
+    oracle.dgbtrs(Ao, ipo, Bo, n, kl, ku)
+    # dgbtrf (AUTO: the run-time compiled factorization) and dgbtrs (window solve, nrhs 3)
+    Ag, ipg, info_g = _gpu_trf(A0.copy(), n, n, kl, ku)
+    assert np.array_equal(info_g, info_o) and np.array_equal(ipg, ipo)
+    assert np.all(same_bits(Ag, Ao))
+    assert np.all(same_bits(_gpu_trs(Ao, ipo, B0.copy(), n, kl, ku), Bo))
+    # dgbtrfs nrhs 1: the library's plan, the two-launch plan and the fused kernel
+    B1 = I.gen_rhs(n, 1, ldb=n + 2, count=batch)
+    B1o = B1.copy()
+    oracle.dgbtrs(Ao, ipo, B1o, n, kl, ku)
+    for phase in (0, bl.TRFS_TWO_LAUNCH, bl.TRFS_FUSED):
+        Ag2, Pg2, Bg2, Ig2 = _trfs(A0.copy(), B1.copy(), n, kl, ku, phase)
+        assert np.array_equal(Ig2, info_o) and np.array_equal(Pg2, ipo)
+        assert np.all(same_bits(Ag2, Ao)) and np.all(same_bits(Bg2, B1o))
+    # dgbsv with a singular matrix: B untouched there
+    As = A0.copy()
+    kv = kl + ku
+    As[5, 40, kl:kv + kl + 1] = np.where(np.isnan(As[5, 40, kl:kv + kl + 1]), np.nan, 0.0)
+    Asv, Bsv = As.copy(), B1.copy()
+    ips, infs = oracle.dgbsv(Asv, Bsv, n, kl, ku)
+    Ag = torch.from_numpy(As).cuda(); Bg = torch.from_numpy(B1.copy()).cuda()
+    P = torch.zeros((batch, n), dtype=torch.int32, device="cuda")
+    inf = torch.zeros(batch, dtype=torch.int32, device="cuda")
+    bl.dgbsv_strided_batched(n, kl, ku, Ag, P, Bg, inf)
+    torch.cuda.synchronize()
+    assert np.array_equal(inf.cpu().numpy(), infs) and infs[5] == 41
+    assert np.all(same_bits(Ag.cpu().numpy(), Asv)) and np.all(same_bits(Bg.cpu().numpy(), Bsv))
+    assert np.all(same_bits(Bg.cpu().numpy()[5], B1[5]))
+
+
+@pytest.mark.parametrize("kl,ku", [(16, 16), (0, 32)])
+def test_jit_band_full_batch_sampled(kl, ku):
+    """A run-time compiled band at a multi-wave batch (the two-launch plan), sampled."""
+    if not bl.jit_band(kl, ku):
+        pytest.skip("NVRTC not available")
+    batch, n = 6000, 256
+    A = torch.from_numpy(I.gen_band(n, n, kl, ku, count=batch)).cuda()
+    B = torch.from_numpy(I.gen_rhs(n, 1, count=batch)).cuda()
+    P = torch.zeros((batch, n), dtype=torch.int32, device="cuda")
+    info = torch.zeros(batch, dtype=torch.int32, device="cuda")
+    bl.dgbtrfs_strided_batched(n, kl, ku, A, P, B, info)
+    torch.cuda.synchronize()
+    for i in _sample_indices(batch, per_warp=(2, 8, 32), extra=16):
+        Ao = I.gen_band(n, n, kl, ku, count=1, first=i)
+        Bo = I.gen_rhs(n, 1, count=1, first=i)
+        ipo, info_o = oracle.dgbtrf(Ao, n, n, kl, ku)
+        oracle.dgbtrs(Ao, ipo, Bo, n, kl, ku)
+        assert np.array_equal(P[i].cpu().numpy(), ipo[0])
+        assert np.all(same_bits(A[i].cpu().numpy(), Ao[0])) and np.all(same_bits(B[i].cpu().numpy(), Bo[0]))
