@@ -1,0 +1,24 @@
+#!/bin/bash
+# Round-2 measurement session: smoke, GPU tests, benches (C3 default + cpu baseline + e2e,
+# reference arm, the other configs, strong-scaling shards), ncu launch list + full captures.
+OUT=gpurun_out; mkdir -p $OUT/prof
+export BANDLU_JIT_CACHE=/tmp/bandlu_jit; mkdir -p $BANDLU_JIT_CACHE
+python -c "import __graft_entry__ as g; g.build(); g.smoke()" > $OUT/smoke.log 2>&1; tail -1 $OUT/smoke.log
+timeout 1200 python -m pytest tests -m gpu -q > $OUT/pytest_gpu.log 2>&1; echo "pytest rc=$?"; tail -1 $OUT/pytest_gpu.log
+python bench.py > $OUT/bench_default.json 2> $OUT/bench_default.err; echo "bench rc=$?"
+python bench.py --impl reference --steps 4 > $OUT/bench_reference.json 2>$OUT/bench_reference.err
+for c in C1 C2 C4 XGC PELE; do timeout 600 python bench.py --config $c --steps 30 --warmup 3 --no-cpu > $OUT/bench_$c.json 2>$OUT/bench_$c.err; done
+for b in 5000 2500 1250; do timeout 600 python bench.py --batch $b --scaling strong --steps 30 --warmup 3 --no-cpu --e2e-steps 0 > $OUT/bench_C3_b$b.json 2>$OUT/bench_C3_b$b.err; done
+python tools/summ.py $OUT/bench_default.json $OUT/bench_C*.json $OUT/bench_XGC.json $OUT/bench_PELE.json
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_c3.csv python bench.py --steps 2 --warmup 3 --e2e-steps 0 --no-cpu > $OUT/ncu_launch_bench.log 2>&1
+for c in C3 C2 C4 C5W; do
+  timeout 900 ncu --set full --clock-control none --import-source on -k regex:gbtr -c 2 -o $OUT/full_$c python tools/prof_step.py $c > $OUT/ncu_full_$c.log 2>&1
+done
+cp profiles/ncu_summary.json $OUT/prof/ 2>/dev/null
+PROF_DIR=$OUT/prof python tools/make_profiles.py r02 C3 C2 C4 C5W > /dev/null
+ncu -i $OUT/full_C3.ncu-rep --page source --csv --print-source sass > $OUT/src_C3.csv 2>/dev/null
+python tools/sass_hist.py $OUT/src_C3.csv 40 > $OUT/prof/sass_hist_C3.txt 2>/dev/null
+ncu -i $OUT/full_C5W.ncu-rep --page source --csv --print-source sass > $OUT/src_C5W.csv 2>/dev/null
+python tools/sass_hist.py $OUT/src_C5W.csv 40 > $OUT/prof/sass_hist_C5W.txt 2>/dev/null
+rm -f $OUT/full_*.ncu-rep $OUT/src_*.csv
+cat $OUT/prof/r02_summary.md | head -60

@@ -15,7 +15,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 OUT = os.path.join(ROOT, "gpurun_out")
 PROF = os.environ.get("PROF_DIR") or os.path.join(ROOT, "profiles")  # the GPU box writes into gpurun_out/
 
-KERNELS = ("gbtrf_rows_kernel", "gbtrf_window_kernel", "gbtrf_wide_kernel", "gbtrf_tc_kernel", "gbtrf_generic_kernel",
+KERNELS = ("gbtrf_tpm_kernel", "gbtrf_rows_kernel", "gbtrf_window_kernel", "gbtrf_wide_kernel", "gbtrf_tc_kernel", "gbtrf_generic_kernel",
            "gbtrs_window_kernel", "gbtrs_bwd_kernel", "gbtrs_rows_kernel", "gbtrs_generic_kernel", "gbtrs_t_generic_kernel")
 KEYS = {
     "duration_us": ("gpu__time_duration.sum", 1e-3),
@@ -102,7 +102,8 @@ def main():
     summary = json.load(open(jpath)) if os.path.exists(jpath) else {}
     md = [f"# ncu summary, round {rnd}", "",
           "Captured with `ncu --set full --clock-control none --import-source on -k regex:gbtr` on one B200",
-          "(`tools/prof_step.py <cfg>`: one dgbtrf + dgbtrs step at the BASELINE config). ncu times are",
+          "(`tools/prof_step.py <cfg>`: one dgbtrfs step -- the library's plan -- at the BASELINE config;",
+          "C5W = C5's (32,32) band at n = 512, batch 4,000). ncu times are",
           "cold-cache and serialised; bench.py numbers come from CUDA events without a profiler.", ""]
     for c in cfgs:
         rep = os.path.join(OUT, f"full_{c}.ncu-rep")

@@ -15,7 +15,8 @@ from paper_conf_sc_abdelfattahtlad23_b200 import inputs as I  # noqa: E402
 
 cfg = sys.argv[1] if len(sys.argv) > 1 else "C3"
 reps = int(sys.argv[2]) if len(sys.argv) > 2 else 1
-bpg, n, kl, ku, nrhs, _ = bench.CONFIGS[cfg]
+EXTRA = {"C5W": (4000, 512, 32, 32, 1, "C5 (32,32) n=512"), "C5N": (20000, 512, 10, 7, 1, "C5 (10,7) n=512")}
+bpg, n, kl, ku, nrhs, _ = EXTRA[cfg] if cfg in EXTRA else bench.CONFIGS[cfg]
 bpg = int(os.environ.get("PROF_BATCH", bpg))
 A0 = I.gen_band_torch(n, n, kl, ku, count=bpg, device='cuda')
 B0 = I.gen_rhs_torch(n, nrhs, count=bpg, device='cuda')
