@@ -237,7 +237,7 @@ def parse(argv=None):
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--parity-sample", type=int, default=24, help="random matrices per rank checked vs the oracle")
     ap.add_argument("--fill", type=float, default=0.3, help="C5: fraction of free HBM per sweep point")
-    ap.add_argument("--plan", default="auto", choices=["auto", "two", "fused"],
+    ap.add_argument("--plan", default="auto", choices=["auto", "two", "fused", "thin"],
                     help="dgbtrfs plan: the library's choice, the two-launch plan (factorization + forward, then "
                          "backward), or the fused single-launch kernel")
     ap.add_argument("--c5-ns", default="", help="C5: comma-separated n list (default 32,64,128..2048 step 128)")
@@ -265,7 +265,7 @@ def run_config(args):
     ldab = 2 * kl + ku + 1
     b_trf, b_trs = I.alg_bytes(n, n, kl, ku, nrhs)
     f_trf, f_trs = I.nominal_flops(n, kl, ku, nrhs)
-    xph = {"auto": 0, "two": bl.TRFS_TWO_LAUNCH, "fused": bl.TRFS_FUSED}[args.plan]
+    xph = {"auto": 0, "two": bl.TRFS_TWO_LAUNCH, "fused": bl.TRFS_FUSED, "thin": bl.TRFS_THIN}[args.plan]
     plan = bl.trfs_plan(n, kl, ku, nrhs, cnt, xph)  # the kernels one dgbtrfs call launches
     per_launch_bytes = [I.alg_bytes_kind(n, kl, ku, nrhs, k) for k in plan["bytes"]]
     big = cnt * n * ldab * 8 > 2 * 126e6
@@ -431,7 +431,7 @@ def run_sweep(args):
             A, B = torch.empty_like(A0), torch.empty_like(B0)
             P = torch.zeros((bpg, n), dtype=torch.int32, device=dev)
             info = torch.zeros(bpg, dtype=torch.int32, device=dev)
-            xph = {"auto": 0, "two": bl.TRFS_TWO_LAUNCH, "fused": bl.TRFS_FUSED}[args.plan]
+            xph = {"auto": 0, "two": bl.TRFS_TWO_LAUNCH, "fused": bl.TRFS_FUSED, "thin": bl.TRFS_THIN}[args.plan]
             plan = bl.trfs_plan(n, kl, ku, 1, bpg, xph)
             nph = len(plan["kernels"])
 

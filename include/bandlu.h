@@ -98,9 +98,12 @@ enum bandlu_variant {
     BANDLU_THREAD = 5,  /* dgbtrf only: one thread per matrix, the whole (kl+1) x (kl+ku+1) window in
                            registers, thin compiled bands (bandlu_thread_available); bitwise equal
                            results */
-    BANDLU_TPM = 6      /* dgbtrf only, square (m == n): one thread per matrix, the window in shared
+    BANDLU_TPM = 6,     /* dgbtrf only, square (m == n): one thread per matrix, the window in shared
                            memory, 4-column panels factored in registers and a rank-4 trailing
                            update per panel (bandlu_tpm_available); bitwise equal results */
+    BANDLU_THIN = 7     /* dgbtrf only, square, strided: thin bands, one thread per matrix with the
+                           window in registers and whole band columns staged cooperatively through
+                           shared memory (bandlu_thin_available); bitwise equal results */
 };
 
 /* ---- dgbtrf: band LU with partial pivoting ---- */
@@ -167,6 +170,7 @@ int dgbtrfs_strided_batched(int n, int kl, int ku, int nrhs,
  * both flags) returns -16. */
 #define BANDLU_TRFS_TWO_LAUNCH 16
 #define BANDLU_TRFS_FUSED 32
+#define BANDLU_TRFS_THIN 64 /* the thin-band thread-per-matrix fused kernel (bandlu_thin_available) */
 int dgbtrfs_strided_batched_ex(int n, int kl, int ku, int nrhs,
                                double *dA, int ldab, int64_t strideA,
                                int *dipiv, int64_t strideP,
@@ -216,6 +220,9 @@ int bandlu_rows_available(int kl, int ku);
 int bandlu_thread_available(int kl, int ku);
 /* 1 if a thread-per-matrix shared-memory-window kernel (BANDLU_TPM) is compiled for (kl, ku), else 0. */
 int bandlu_tpm_available(int kl, int ku);
+/* 1 if a thin-band thread-per-matrix kernel (BANDLU_THIN) is compiled for (kl, ku), else 0
+ * (only in -DBANDLU_WITH_THIN builds: measured slower, AUTO never picks it). */
+int bandlu_thin_available(int kl, int ku);
 /* Run-time compiled bands (Sec. 8.1: JIT-compiled register-resident
  * kernels).  A (kl, ku) that no ahead-of-time instantiation covers takes the same kernel
  * templates compiled with NVRTC for sm_100a on the first call that needs them (seconds;
@@ -235,10 +242,10 @@ int bandlu_trs_rows_available(int kl, int ku);
  * returns their number L (0..2; < 0 on a negative argument) and, if kinds is
  * not NULL, writes L codes kinds[i] = 16 * kernel + bytes, kernel: 1 gbtrf_rows,
  * 2 gbtrf_window, 3 gbtrf_wide, 4 gbtrf_thread, 5 gbtrf_generic, 6 gbtrs_bwd,
- * 7 gbtrs_rows, 8 gbtrs_window, 9 gbtrs_generic; bytes (what the launch must
+ * 7 gbtrs_rows, 8 gbtrs_window, 9 gbtrs_generic, 10 gbtrf_thin; bytes (what the launch must
  * move per matrix): 1 factorization, 2 factorization + forward
  * substitution, 3 backward substitution, 4 full solve, 5 fused gbsv.
- * phase: 0, BANDLU_TRFS_TWO_LAUNCH or BANDLU_TRFS_FUSED (as for dgbtrfs). */
+ * phase: 0, BANDLU_TRFS_TWO_LAUNCH, BANDLU_TRFS_FUSED or BANDLU_TRFS_THIN (as for dgbtrfs). */
 int bandlu_trfs_plan(int n, int kl, int ku, int nrhs, int batch, int phase, int *kinds);
 /* ABI version of this library. */
 int bandlu_version(void);

@@ -18,7 +18,7 @@ import torch
 
 from . import _build
 
-AUTO, GENERIC, WINDOW, TC, ROWS, THREAD, TPM = 0, 1, 2, 3, 4, 5, 6
+AUTO, GENERIC, WINDOW, TC, ROWS, THREAD, TPM, THIN = 0, 1, 2, 3, 4, 5, 6, 7
 ERR_UNSUPPORTED, ERR_CUDA = 1000, 2000
 
 _lib = None
@@ -72,6 +72,7 @@ def load(build_if_missing: bool = False):
         "bandlu_trs_rows_available": [i, i],
         "bandlu_thread_available": [i, i],
         "bandlu_tpm_available": [i, i],
+        "bandlu_thin_available": [i, i],
         "bandlu_jit_band": [i, i],
         "bandlu_jit_check": [i, i, p, i],
         "bandlu_trs_variant": [i, i, i, i],
@@ -90,7 +91,7 @@ def load(build_if_missing: bool = False):
 EXPORTS = ("dgbtrf_batched", "dgbtrf_strided_batched", "dgbtrf_strided_batched_ex", "dgbtrs_batched",
            "dgbtrs_strided_batched", "dgbtrs_strided_batched_ex", "dgbsv_batched", "dgbsv_strided_batched",
            "dgbsv_strided_batched_host", "dgbtrfs_strided_batched", "dgbtrfs_strided_batched_ex", "bandlu_trf_variant", "bandlu_trs_variant", "bandlu_tc_available", "bandlu_rows_available", "bandlu_trs_rows_available", "bandlu_thread_available",
-           "bandlu_tpm_available", "bandlu_jit_band", "bandlu_jit_check", "bandlu_trfs_plan", "bandlu_version")
+           "bandlu_tpm_available", "bandlu_thin_available", "bandlu_jit_band", "bandlu_jit_check", "bandlu_trfs_plan", "bandlu_version")
 
 
 def _stream(stream):
@@ -252,6 +253,11 @@ def tpm_available(kl: int, ku: int) -> bool:
     return bool(load().bandlu_tpm_available(kl, ku))
 
 
+def thin_available(kl: int, ku: int) -> bool:
+    """True if the thin-band thread-per-matrix kernel (variant THIN) is compiled for (kl, ku)."""
+    return bool(load().bandlu_thin_available(kl, ku))
+
+
 def jit_band(kl: int, ku: int) -> bool:
     """True if (kl, ku) is served by run-time compiled (NVRTC) kernels (include/bandlu.h)."""
     return bool(load().bandlu_jit_band(kl, ku))
@@ -275,9 +281,9 @@ def trs_variant(n: int, kl: int, ku: int, nrhs: int) -> int:
 
 KERNEL_NAMES = {1: "gbtrf_rows_kernel", 2: "gbtrf_window_kernel", 3: "gbtrf_wide_kernel", 4: "gbtrf_thread_kernel",
                 5: "gbtrf_generic_kernel", 6: "gbtrs_bwd_kernel", 7: "gbtrs_rows_kernel", 8: "gbtrs_window_kernel",
-                9: "gbtrs_generic_kernel"}
+                9: "gbtrs_generic_kernel", 10: "gbtrf_thin_kernel"}
 BYTE_KINDS = {1: "trf", 2: "trf_fwd", 3: "trs_bwd", 4: "trs", 5: "gbsv"}
-TRFS_TWO_LAUNCH, TRFS_FUSED = 16, 32
+TRFS_TWO_LAUNCH, TRFS_FUSED, TRFS_THIN = 16, 32, 64
 
 
 def trfs_plan(n: int, kl: int, ku: int, nrhs: int, batch: int, phase: int = 0) -> dict:

@@ -18,6 +18,7 @@
 #include "gbtrf_wide.cuh"
 #include "gbtrf_tc.cuh"
 #include "gbtrf_thread.cuh"
+#include "gbtrf_thin.cuh"
 #include "gbtrf_tpm.cuh"
 #include "gbtrf_window.cuh"
 #include "gbtrs_bwd.cuh"
@@ -103,6 +104,26 @@ namespace {
 #define BANDLU_TPM_LIST(X) X(10, 10, BANDLU_TPM_MPW)
 #else
 #define BANDLU_TPM_LIST(X)
+#endif
+
+// (KL, KU) compiled as thin-band thread-per-matrix kernels with cooperative whole-column
+// staging (gbtrf_thin.cuh; square matrices).  Opt-in experiment (-DBANDLU_WITH_THIN): bitwise
+// equal, but measured slower than the row-slot kernels -- C2 one-launch 0.483 vs 0.242 ms, C2
+// factorization 0.318 vs 0.145 ms, C1 0.174 vs 0.035 ms
+#if !defined(BANDLU_WITH_THIN)
+#define BANDLU_THIN_LIST(X)
+#elif defined(BANDLU_ONLY_C3)
+#define BANDLU_THIN_LIST(X) X(1, 1)
+#else
+#define BANDLU_THIN_LIST(X) \
+    X(0, 0)                 \
+    X(0, 3)                 \
+    X(1, 1)                 \
+    X(2, 2)                 \
+    X(2, 3)                 \
+    X(3, 0)                 \
+    X(3, 2)                 \
+    X(4, 4)
 #endif
 
 // (KL, KU) compiled as thread-per-matrix factorization kernels (gbtrf_thread.cuh, thin
@@ -220,6 +241,26 @@ int launch_trf_thread(int m, int n, AP A, int ldab, PP P, int *info, int batch, 
     if (int r = set_smem(k, C::smem_bytes())) return r;
     k<<<grid, C::THREADS, C::smem_bytes(), st>>>(m, n, A, ldab, P, info, batch, B);
     return cuda_ret(cudaGetLastError());
+}
+
+template <int KL, int KU, int FL, class AP, class PP, class BP>
+int launch_trf_thin(int n, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st, BP B) {
+    using C = TrfThin<KL, KU>;
+    auto k = gbtrf_thin_kernel<KL, KU, FL, AP, PP, BP>;
+    const size_t sm = C::smem_bytes(ldab);
+    if (sm > 227 * 1024) return BANDLU_ERR_UNSUPPORTED;
+    if (int r = set_smem(k, sm)) return r;
+    const unsigned grid = (unsigned)((batch + 31) / 32);
+    k<<<grid, 32, sm, st>>>(n, A, ldab, P, info, batch, B);
+    return cuda_ret(cudaGetLastError());
+}
+
+bool trf_thin_available(int kl, int ku) {
+#define X(a, b) \
+    if (kl == a && ku == b) return true;
+    BANDLU_THIN_LIST(X)
+#undef X
+    return false;
 }
 
 template <int KL, int KU, int MPW, bool FWD, class AP, class PP, class BP>
@@ -419,6 +460,16 @@ int run_trf(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int b
 #undef X
         return BANDLU_ERR_UNSUPPORTED;
     }
+    if (variant == BANDLU_THIN && m > 0 && n > 0) {
+        if (m != n) return BANDLU_ERR_UNSUPPORTED;
+        if constexpr (std::is_same_v<AP, Strided<double>>) {
+#define X(a, b) \
+    if (kl == a && ku == b) return launch_trf_thin<a, b, 0>(n, A, ldab, P, info, batch, st, Strided<double>{nullptr, 0});
+            BANDLU_THIN_LIST(X)
+#undef X
+        }
+        return BANDLU_ERR_UNSUPPORTED;
+    }
     if (variant == BANDLU_TPM && m > 0 && n > 0) {
         if (m != n) return BANDLU_ERR_UNSUPPORTED;
 #define X(a, b, w) \
@@ -462,7 +513,7 @@ int run_trf(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int b
         return BANDLU_ERR_UNSUPPORTED;
     }
     if (variant != BANDLU_GENERIC && variant != BANDLU_WINDOW && variant != BANDLU_TC && variant != BANDLU_ROWS &&
-        variant != BANDLU_THREAD && variant != BANDLU_TPM)
+        variant != BANDLU_THREAD && variant != BANDLU_TPM && variant != BANDLU_THIN)
         return BANDLU_ERR_UNSUPPORTED;
     return launch_trf_generic(m, n, kl, ku, A, ldab, P, info, batch, st);
 }
@@ -622,7 +673,7 @@ int launch_trs_bwd(int n, AP A, int ldab, PP P, BP B, int ldb, int batch, cudaSt
 // solves B even where info > 0; dgbsv leaves B untouched there).
 // phase: 0 = every launch, 1 = first launch only, 2 = second launch only (the
 // bench times them separately); | TRFS_TWO_LAUNCH forces the two-launch plan.
-constexpr int TRFS_TWO_LAUNCH = BANDLU_TRFS_TWO_LAUNCH, TRFS_FUSED = BANDLU_TRFS_FUSED;
+constexpr int TRFS_TWO_LAUNCH = BANDLU_TRFS_TWO_LAUNCH, TRFS_FUSED = BANDLU_TRFS_FUSED, TRFS_THIN = BANDLU_TRFS_THIN;
 constexpr size_t kSmemPerSM = 227 * 1024;
 
 template <int KL, int KU, int G, int R>
@@ -680,7 +731,7 @@ bool rows_ysm_fits_rt(int n, int kl, int ku) {
 
 // kernel ids / byte classes reported by bandlu_trfs_plan (include/bandlu.h)
 enum { KN_TRF_ROWS = 1, KN_TRF_WINDOW, KN_TRF_WIDE, KN_TRF_THREAD, KN_TRF_GENERIC, KN_TRS_BWD, KN_TRS_ROWS,
-       KN_TRS_WINDOW, KN_TRS_GENERIC };
+       KN_TRS_WINDOW, KN_TRS_GENERIC, KN_TRF_THIN };
 enum { KB_TRF = 1, KB_TRF_FWD, KB_TRS_BWD, KB_TRS, KB_GBSV };
 
 // run-time compiled bands, nrhs == 1: is the fused kernel picked?  (geometry from the
@@ -699,6 +750,11 @@ int trfs_plan(int n, int kl, int ku, int nrhs, int64_t batch, int phase, int *ki
     int k = 0;
     auto put = [&](int name, int bytes) { if (kinds) kinds[k] = name * 16 + bytes; ++k; };
     if (n <= 0 || nrhs <= 0) return 0;
+    if ((phase & TRFS_THIN) && nrhs == 1 && trf_thin_available(kl, ku)) {
+        put(KN_TRF_THIN, KB_GBSV);
+        return k;
+    }
+    phase &= ~TRFS_THIN;
     if (nrhs == 1 && jit_band(kl, ku)) {
         const bandlu_jit::Kern &K = jit_trf(kl, ku, FL_FWD);
         if (K.ok) {
@@ -735,10 +791,18 @@ int trfs_plan(int n, int kl, int ku, int nrhs, int64_t batch, int phase, int *ki
 template <class AP, class PP, class BP>
 int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ldb, int *info, int batch,
              cudaStream_t st, int phase) {
+    if (batch == 0) return 0;
+    if ((phase & TRFS_THIN) && n > 0 && nrhs == 1 && trf_thin_available(kl, ku)) {
+        if ((phase & 3) == 2) return 0;  // one launch
+#define X(a, b) \
+    if (kl == a && ku == b) return launch_trf_thin<a, b, 3>(n, A, ldab, P, info, batch, st, B);
+        BANDLU_THIN_LIST(X)
+#undef X
+    }
+    phase &= ~TRFS_THIN;
     const bool fused = trfs_fused_pick(n, kl, ku, nrhs, batch, phase);
     const int pflags = phase & (TRFS_TWO_LAUNCH | TRFS_FUSED);
     phase &= ~(TRFS_TWO_LAUNCH | TRFS_FUSED);
-    if (batch == 0) return 0;
     if (fused) {
         if (phase == 2) return 0;  // the whole path is the first (only) launch
         const bool ysm = rows_ysm_fits_rt(n, kl, ku);
@@ -926,6 +990,7 @@ int bandlu_tc_available(int kl, int ku) { return trf_tc_available(kl, ku) ? 1 : 
 int bandlu_rows_available(int kl, int ku) { return trf_rows_available(kl, ku) ? 1 : 0; }
 int bandlu_thread_available(int kl, int ku) { return trf_thread_available(kl, ku) ? 1 : 0; }
 int bandlu_tpm_available(int kl, int ku) { return trf_tpm_available(kl, ku) ? 1 : 0; }
+int bandlu_thin_available(int kl, int ku) { return trf_thin_available(kl, ku) ? 1 : 0; }
 
 // 1 if (kl, ku) is served by run-time compiled kernels (jit.cuh), else 0 (no compilation)
 int bandlu_jit_band(int kl, int ku) { return jit_band(kl, ku) ? 1 : 0; }
@@ -965,7 +1030,7 @@ int bandlu_trs_variant(int n, int kl, int ku, int nrhs) { return pick_trs(n, kl,
 int bandlu_trfs_plan(int n, int kl, int ku, int nrhs, int batch, int phase, int *kinds) {
     if (n < 0 || kl < 0 || ku < 0 || nrhs < 0 || batch < 0) return -1;
     if ((phase & TRFS_TWO_LAUNCH) && (phase & TRFS_FUSED)) return -1;
-    return trfs_plan(n, kl, ku, nrhs, batch, phase, kinds);
+    return trfs_plan(n, kl, ku, nrhs, batch, phase, kinds);  // phase flags as for dgbtrfs
 }
 
 int dgbtrf_strided_batched_ex(int m, int n, int kl, int ku, double *dA, int ldab, int64_t strideA, int *dipiv,
@@ -1058,7 +1123,10 @@ int dgbtrfs_strided_batched_ex(int n, int kl, int ku, int nrhs, double *dA, int 
         if (!dinfo) return -13;
     }
     if ((phase & TRFS_TWO_LAUNCH) && (phase & TRFS_FUSED)) return -16;
-    if ((phase & ~(TRFS_TWO_LAUNCH | TRFS_FUSED)) < 0 || (phase & ~(TRFS_TWO_LAUNCH | TRFS_FUSED)) > 2) return -16;
+    {
+        const int ph = phase & ~(TRFS_TWO_LAUNCH | TRFS_FUSED | TRFS_THIN);
+        if (ph < 0 || ph > 2) return -16;
+    }
     return run_trfs(n, kl, ku, nrhs, Strided<double>{dA, strideA}, ldab, Strided<int>{dipiv, strideP},
                     Strided<double>{dB, strideB}, ldb, dinfo, batch, (cudaStream_t)stream, phase);
 }

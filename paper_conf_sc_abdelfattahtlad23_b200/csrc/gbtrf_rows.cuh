@@ -29,6 +29,9 @@
 #pragma once
 #include "backsolve_fused.cuh"
 #include "common.cuh"
+#ifndef __CUDACC_RTC__
+#include <type_traits>
+#endif
 
 #ifndef BANDLU_ROWS_WARPS
 #define BANDLU_ROWS_WARPS 4
@@ -43,8 +46,14 @@ struct TrfRows {
 #ifndef BANDLU_ROWS_U
 #define BANDLU_ROWS_U 4
 #endif
-    static constexpr int U = BANDLU_ROWS_U;      // columns per block (window shift granularity)
-    static constexpr int WS = W + U, H = (WS + 1) / 2;
+    static constexpr int U = BANDLU_ROWS_U;      // columns per block (preload / record granularity)
+#ifndef BANDLU_ROWS_NBLK
+#define BANDLU_ROWS_NBLK 1
+#endif
+    // blocks per register-window shift: with 2 the window holds NBLK*U extra columns and the
+    // second block of a pair addresses its slots U further on, halving the shift moves
+    static constexpr int NBLK = BANDLU_ROWS_NBLK;
+    static constexpr int WS = W + NBLK * U, H = (WS + 1) / 2;
     static_assert(G * R >= KL + 1 + U, "slots: KL+1 active rows + U preloaded rows");
     static_assert(32 % G == 0, "group size");
     // ring row / record pitch (doubles), spare pair at RP: (B entry[, logical row])
@@ -295,8 +304,9 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
         o.rb = rb;
         o.gb = gb;
     };
-#pragma unroll 1
-    for (int j0 = 0; j0 < mn; j0 += U) {
+    // one block of U columns; its column j0+s sits in register slot OFF+s
+    auto blk = [&](auto offc, int j0) {
+        constexpr int OFF = decltype(offc)::value;
         cp_async_wait<C::DB - 1>();  // rows j0+KL+1 .. j0+KL+U landed (this lane's part)
         __syncwarp();
         // ---- preload rows j0+KL+1+o (o = 0..U-1) into the first U free slots of the group
@@ -311,7 +321,7 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
                 const int q = j0 + KL + 1 + rank;
                 const uint32_t rr = ring_s + (uint32_t)((q & (RR - 1)) * WP * 8);
 #pragma unroll
-                for (int h = 0; h < H; ++h) ld_shared_v2_if(take, rr + h * 16, v[ri][h]);
+                for (int h = 0; h < H - OFF / 2; ++h) ld_shared_v2_if(take, rr + h * 16, v[ri][h + OFF / 2]);
                 if constexpr (FWD) ld_shared_f64_if(take, rr + RP * 8, bq[ri]);
                 if (take) pos[ri] = q;
                 before += __popc(fb);
@@ -326,7 +336,7 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
 
             // ---- IAMAX over the candidates (logical rows j..min(j+KL, m-1)); with LOOKAHEAD
             // the search of step s > 0 already ran inside step s-1, right after column j's update
-            if (!LA || s == 0) search(s, j, ps);
+            if (!LA || s == 0) search(s + OFF, j, ps);
             double x[R];
             bool cand[R];
 #pragma unroll
@@ -346,11 +356,11 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
             // the stall samples, yet removing it measured 0.2341 vs 0.2343 ms (and 0.968 vs
             // 0.960 ms at 10,000): the step time is its instruction count, not that chain.
             const int plane = (int)gbase + max(__ffs(gb) - 1, 0);
-            double xs = x[0], u1s = VS(0, s + 1);
+            double xs = x[0], u1s = VS(0, s + 1 + OFF);
 #pragma unroll
             for (int ri = 1; ri < R; ++ri) {
                 xs = (rb == ri) ? x[ri] : xs;
-                u1s = (rb == ri) ? VS(ri, s + 1) : u1s;
+                u1s = (rb == ri) ? VS(ri, s + 1 + OFF) : u1s;
             }
             const double rinv = __shfl_sync(0xffffffffu, drcp_rn_nz(xs), plane);
             const double u1 = __shfl_sync(0xffffffffu, u1s, plane);
@@ -362,7 +372,8 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
 #pragma unroll
             for (int ri = 0; ri < R; ++ri) {
 #pragma unroll
-                for (int h = s / 2; h <= (s + KV) / 2; ++h) st_shared_v2_if(is_piv && rb == ri, rcs + h * 16, v[ri][h]);
+                for (int h = s / 2; h <= (s + KV) / 2; ++h)
+                    st_shared_v2_if(is_piv && rb == ri, rcs + h * 16, v[ri][h + OFF / 2]);
             }
             {
                 double bsel = bq[0];
@@ -450,19 +461,20 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
 #endif
 #pragma unroll
                 for (int ri = 0; ri < R; ++ri) {
-                    if (2 * h >= s + 1) VS(ri, 2 * h) = __fma_rn(lu[ri], -ua, VS(ri, 2 * h));
-                    if (2 * h + 1 <= s + KV) VS(ri, 2 * h + 1) = __fma_rn(lu[ri], -ub, VS(ri, 2 * h + 1));
+                    if (2 * h >= s + 1) VS(ri, 2 * h + OFF) = __fma_rn(lu[ri], -ua, VS(ri, 2 * h + OFF));
+                    if (2 * h + 1 <= s + KV)
+                        VS(ri, 2 * h + 1 + OFF) = __fma_rn(lu[ri], -ub, VS(ri, 2 * h + 1 + OFF));
                 }
                 // column j+1 (slot s+1) is final for step j+1: its pivot search overlaps the
                 // rest of this update
-                if (LA && h == (s + 1) / 2 && s + 1 < U && j + 1 < mn) search(s + 1, j + 1, ps);
+                if (LA && h == (s + 1) / 2 && s + 1 < U && j + 1 < mn) search(s + 1 + OFF, j + 1, ps);
             }
 #else
 #pragma unroll
             for (int k = 1; k <= KV; ++k) {
                 const double uk = ld_volatile_shared_f64(rcs + (s + k) * 8);
 #pragma unroll
-                for (int ri = 0; ri < R; ++ri) VS(ri, s + k) = __fma_rn(lu[ri], -uk, VS(ri, s + k));
+                for (int ri = 0; ri < R; ++ri) VS(ri, s + k + OFF) = __fma_rn(lu[ri], -uk, VS(ri, s + k + OFF));
             }
 #endif
 #pragma unroll
@@ -520,11 +532,19 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
         }
 #endif
         __syncwarp();
-        // shift the window by U columns: slot r <- slot r+U
+    };
+#pragma unroll 1
+    for (int j0 = 0; j0 < mn; j0 += C::NBLK * U) {
+        blk(std::integral_constant<int, 0>{}, j0);
+        if constexpr (C::NBLK == 2) {
+            if (j0 + U < mn) blk(std::integral_constant<int, U>{}, j0 + U);
+        }
+        // shift the window by NBLK*U columns: slot r <- slot r+NBLK*U
+        constexpr int SH = C::NBLK * U;
 #pragma unroll
         for (int ri = 0; ri < R; ++ri) {
 #pragma unroll
-            for (int k = 0; k < 2 * H; ++k) VS(ri, k) = (k + U < 2 * H) ? VS(ri, k + U) : 0.0;
+            for (int k = 0; k < 2 * H; ++k) VS(ri, k) = (k + SH < 2 * H) ? VS(ri, k + SH) : 0.0;
         }
     }
     cp_async_wait<0>();

@@ -43,6 +43,8 @@ def trf_variants(kl, ku, square=True):
     v = [bl.WINDOW, bl.GENERIC] if (kl, ku) in WINDOW_BANDS else [bl.GENERIC]
     if square and bl.tpm_available(kl, ku):
         v.append(bl.TPM)
+    if square and bl.thin_available(kl, ku):
+        v.append(bl.THIN)
     if bl.rows_available(kl, ku):
         v.append(bl.ROWS)
     if bl.tc_available(kl, ku):
@@ -65,7 +67,7 @@ def _check_trf(m, n, kl, ku, batch, variant, ldab=None, first=0, A_in=None):
 
 
 @pytest.mark.parametrize("kl,ku", ALL_BANDS)
-@pytest.mark.parametrize("variant", [bl.WINDOW, bl.GENERIC, bl.ROWS, bl.TC, bl.THREAD, bl.TPM])
+@pytest.mark.parametrize("variant", [bl.WINDOW, bl.GENERIC, bl.ROWS, bl.TC, bl.THREAD, bl.TPM, bl.THIN])
 @pytest.mark.parametrize("n", [1, 2, 7, 37, 100])
 def test_trf_parity_small(kl, ku, variant, n):
     if variant not in trf_variants(kl, ku):
@@ -585,3 +587,37 @@ def test_jit_band_full_batch_sampled(kl, ku):
         oracle.dgbtrs(Ao, ipo, Bo, n, kl, ku)
         assert np.array_equal(P[i].cpu().numpy(), ipo[0])
         assert np.all(same_bits(A[i].cpu().numpy(), Ao[0])) and np.all(same_bits(B[i].cpu().numpy(), Bo[0]))
+
+
+
+# ------------------------------------------------ thin bands, thread per matrix
+THIN_BANDS = [(0, 0), (0, 3), (1, 1), (2, 2), (2, 3), (3, 0), (3, 2), (4, 4)]
+
+
+@pytest.mark.parametrize("kl,ku", THIN_BANDS)
+@pytest.mark.parametrize("n", [1, 2, 7, 8, 9, 33, 150])
+def test_thin_fused_kernel_vs_oracle(kl, ku, n):
+    """The thin-band kernel's one-launch dgbtrf + dgbtrs (cooperative whole-column staging,
+    forward and backward passes by the owning thread) equals the oracle bitwise: n below,
+    at and around the block of 8 columns, a ragged batch (a partly empty last warp), a
+    singular matrix (B solved regardless, as dgbtrfs specifies) and padded ldab / ldb."""
+    if not bl.thin_available(kl, ku):
+        pytest.skip("no thin kernel for this band")
+    batch = 45
+    for ldab in (None, 2 * kl + ku + 1 + 3):
+        A = I.gen_band(n, n, kl, ku, ldab=ldab, count=batch, first=n)
+        if n > 4:
+            kv = kl + ku
+            lo, hi = kl, kv + kl + 1
+            A[6, 3, lo:hi] = np.where(np.isnan(A[6, 3, lo:hi]), np.nan, 0.0)
+        B = I.gen_rhs(n, 1, ldb=n + 2, count=batch)
+        Ao, Bo = A.copy(), B.copy()
+        ipo, info_o = oracle.dgbtrf(Ao, n, n, kl, ku)
+        oracle.dgbtrs(Ao, ipo, Bo, n, kl, ku)
+        Ag, Pg, Bg, Ig = _trfs(A.copy(), B.copy(), n, kl, ku, bl.TRFS_THIN)
+        assert np.array_equal(Ig, info_o) and np.array_equal(Pg, ipo)
+        assert np.all(same_bits(Ag, Ao))  # incl. NaN corners / padding rows
+        ok = same_bits(Bg, Bo)
+        if n > 4:
+            ok[6] = True  # singular U: Inf/NaN pattern of x out of contract (reading 12)
+        assert np.all(ok)
