@@ -73,3 +73,23 @@ def test_torch_generator_matches_numpy_generator():
     r = I.gen_rhs(50, 3, ldb=53, count=4, first=99)
     t = I.gen_rhs_torch(50, 3, count=4, first=99, ldb=53).numpy()
     assert np.array_equal(np.isnan(r), np.isnan(t)) and np.array_equal(np.nan_to_num(r), np.nan_to_num(t))
+
+
+def test_bench_parity_checker_catches_a_flipped_bit():
+    """bench.py's post-timing parity check (oracle on runs of sampled matrices) reports 0
+    mismatches for correct outputs and flags a one-ulp change in one factor entry."""
+    import numpy as np
+    sys.path.insert(0, ROOT)
+    import bench
+    import oracle
+    from paper_conf_sc_abdelfattahtlad23_b200 import inputs as I
+    n, kl, ku = 40, 3, 2
+    loc = bench.sample_local(300, 24)
+    assert 0 in loc and 299 in loc and len(loc) >= 24
+    A = np.concatenate([I.gen_band(n, n, kl, ku, count=1, first=i) for i in loc])
+    B = np.concatenate([I.gen_rhs(n, 1, count=1, first=i) for i in loc])
+    ip, inf = oracle.dgbtrf(A, n, n, kl, ku)
+    oracle.dgbtrs(A, ip, B, n, kl, ku)
+    assert bench.parity_check(loc, (A, ip, B, inf), n, kl, ku, 1) == 0
+    A[3, 5, 5] = np.nextafter(A[3, 5, 5], np.inf)
+    assert bench.parity_check(loc, (A, ip, B, inf), n, kl, ku, 1) == 1
