@@ -120,7 +120,11 @@ int dgbtrf_strided_batched(int m, int n, int kl, int ku,
  * identical for real data) with the dgbtrf factors (transA).
  * LAPACK DGBTRS semantics: no singularity check (singular U gives Inf/NaN).
  * 'T' follows the reference-BLAS operation order of DTBSV('U','T') and
- * DGEMV('T') (dot products accumulated in increasing index order). */
+ * DGEMV('T') (dot products accumulated in increasing index order).  For
+ * 'T', AUTO and BANDLU_WINDOW run the ring-staged transposed solve (lane per
+ * (matrix, RHS column); compiled bands, others compiled at run time when
+ * kl + ku <= 64); BANDLU_GENERIC runs one thread per (matrix, RHS column).
+ * Both give bitwise the same result. */
 int dgbtrs_batched(char trans, int n, int kl, int ku, int nrhs,
                    const double *const *dA_array, int ldab,
                    const int *const *dipiv_array,

@@ -23,6 +23,7 @@
 #include "gbtrf_window.cuh"
 #include "gbtrs_bwd.cuh"
 #include "gbtrs_rows.cuh"
+#include "gbtrs_t.cuh"
 #include "gbtrs_window.cuh"
 #include "generic.cuh"
 #include "jit.cuh"
@@ -186,6 +187,10 @@ namespace {
 #define BANDLU_TRS_WPSM 8
 #endif
 constexpr int64_t kTrsWarpsTarget = 148 * BANDLU_TRS_WPSM;
+#ifndef BANDLU_TRST_WPSM
+#define BANDLU_TRST_WPSM BANDLU_TRS_WPSM
+#endif
+constexpr int64_t kTrsTWarpsTarget = 148 * BANDLU_TRST_WPSM;  // transposed solve (gbtrs_t.cuh)
 
 inline int cuda_ret(cudaError_t e) { return e == cudaSuccess ? 0 : BANDLU_ERR_CUDA + (int)e; }
 
@@ -589,12 +594,66 @@ int launch_trs_t_generic(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, 
     return cuda_ret(cudaGetLastError());
 }
 
+// ring-staged transposed solve (gbtrs_t.cuh), lane per (matrix, RHS column) as the window solve
+template <int KL, int KU, class AP, class PP, class BP>
+int launch_trs_t(int n, int nrhs, AP A, int ldab, PP P, BP B, int ldb, int batch, cudaStream_t st) {
+    using C = TrsT<KL, KU>;
+    const int R = nrhs >= 32 ? 32 : pow2_ceil(nrhs);
+    const int chunks = (nrhs + 31) / 32;
+    auto k = gbtrs_t_kernel<KL, KU, AP, PP, BP>;
+    const int64_t units = (int64_t)batch * chunks;
+    int gpw = 32 / R;
+    while (gpw > 1 && units < (int64_t)gpw * kTrsTWarpsTarget) gpw >>= 1;
+    const size_t sm = C::smem_bytes(R, gpw);
+    if (int r = set_smem(k, sm)) return r;
+    const unsigned grid = (unsigned)((units + gpw - 1) / gpw);
+    k<<<grid, 32, sm, st>>>(n, nrhs, A, ldab, P, B, ldb, batch, R, chunks, gpw);
+    return cuda_ret(cudaGetLastError());
+}
+// run-time compiled transposed solve (bands without a compiled one)
+int jit_launch_trs_t(int kl, int ku, int n, int nrhs, Strided<const double> A, int ldab, Strided<const int> P,
+                     Strided<double> B, int ldb, int batch, cudaStream_t st) {
+    int R = nrhs >= 32 ? 32 : pow2_ceil(nrhs);
+    int chunks = (nrhs + 31) / 32;
+    const bandlu_jit::Kern &K = bandlu_jit::trst(kl, ku);
+    if (!K.ok) return BANDLU_ERR_UNSUPPORTED;
+    const int64_t units = (int64_t)batch * chunks;
+    int gpw = 32 / R;
+    while (gpw > 1 && units < (int64_t)gpw * kTrsTWarpsTarget) gpw >>= 1;
+    int li = 0;
+    while ((1 << li) < R) ++li;
+    const size_t sm = (size_t)(K.geo[0] + (long long)gpw * K.geo[1 + li]) * 8;
+    if (sm > 48 * 1024) {
+        cudaError_t e = cudaFuncSetAttribute((const void *)K.k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+        if (e != cudaSuccess) return cuda_ret(e);
+    }
+    const unsigned grid = (unsigned)((units + gpw - 1) / gpw);
+    void *args[] = {&n, &nrhs, &A, &ldab, &P, &B, &ldb, &batch, &R, &chunks, &gpw};
+    return cuda_ret(cudaLaunchKernel((const void *)K.k, dim3(grid), dim3(32), args, sm, st));
+}
+
 template <class AP, class PP, class BP>
 int run_trs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ldb, const int *skip, int batch,
             cudaStream_t st, int variant, char trans = 'N') {
     if (batch == 0 || n == 0 || nrhs == 0) return 0;
     if (trans != 'N' && trans != 'n') {  // A^T X = B ('C' == 'T' for real data)
-        if (variant != BANDLU_AUTO && variant != BANDLU_GENERIC) return BANDLU_ERR_UNSUPPORTED;
+        if (variant == BANDLU_AUTO) variant = (trs_window_available(kl, ku) || jit_trs_band(kl, ku)) ? BANDLU_WINDOW
+                                                                                                     : BANDLU_GENERIC;
+        if (variant == BANDLU_WINDOW) {
+#define X(a, b) \
+    if (kl == a && ku == b) return launch_trs_t<a, b>(n, nrhs, A, ldab, P, B, ldb, batch, st);
+            BANDLU_TRS_LIST(X)
+#undef X
+            if (jit_trs_band(kl, ku)) {
+                if constexpr (std::is_same_v<AP, Strided<const double>>) {
+                    const int r = jit_launch_trs_t(kl, ku, n, nrhs, A, ldab, P, B, ldb, batch, st);
+                    if (r != BANDLU_ERR_UNSUPPORTED) return r;
+                }
+                return launch_trs_t_generic(n, kl, ku, nrhs, A, ldab, P, B, ldb, batch, st);
+            }
+            return BANDLU_ERR_UNSUPPORTED;
+        }
+        if (variant != BANDLU_GENERIC) return BANDLU_ERR_UNSUPPORTED;
         return launch_trs_t_generic(n, kl, ku, nrhs, A, ldab, P, B, ldb, batch, st);
     }
     if (variant == BANDLU_AUTO) variant = pick_trs(n, kl, ku, nrhs);

@@ -364,6 +364,43 @@ def test_trs_transposed_parity(kl, ku, nrhs, trans):
     assert np.all(same_bits(Bg.cpu().numpy(), Bo))
 
 
+# ring-staged transposed solve (gbtrs_t.cuh; compiled bands and a run-time compiled one):
+# n below / at / just above kl and kv (the truncated dot products run outside the ring),
+# nrhs spanning 1, a partial lane group, and two 32-column chunks, ragged batches
+@pytest.mark.parametrize("kl,ku", [(10, 10), (2, 32), (1, 1), (0, 3), (3, 0), (32, 32), (5, 9)])
+@pytest.mark.parametrize("n,nrhs,batch", [(1, 1, 5), (3, 2, 7), (11, 1, 13), (21, 3, 9), (22, 1, 33),
+                                          (160, 1, 301), (97, 5, 41), (70, 33, 6)])
+def test_trs_transposed_ring_kernel(kl, ku, n, nrhs, batch):
+    A = I.gen_band(n, n, kl, ku, count=batch)
+    ipiv, info = oracle.dgbtrf(A, n, n, kl, ku)
+    B = I.gen_rhs(n, nrhs, ldb=n + 1, count=batch)
+    Bo = B.copy()
+    oracle.dgbtrs(A, ipiv, Bo, n, kl, ku, trans="T")
+    Ag = torch.from_numpy(A).cuda(); Pg = torch.from_numpy(ipiv).cuda()
+    for variant in (bl.WINDOW, bl.GENERIC):
+        Bg = torch.from_numpy(B).cuda()
+        bl.dgbtrs_strided_batched("T", n, kl, ku, Ag, Pg, Bg, variant=variant)
+        torch.cuda.synchronize()
+        assert np.all(same_bits(Bg.cpu().numpy(), Bo)), variant  # incl. the NaN padding row of ldb
+
+
+def test_trs_transposed_pointer_array():
+    n, kl, ku, nrhs, batch = 60, 10, 10, 2, 11
+    A = I.gen_band(n, n, kl, ku, count=batch)
+    ipiv, info = oracle.dgbtrf(A, n, n, kl, ku)
+    B = I.gen_rhs(n, nrhs, count=batch)
+    Bo = B.copy()
+    oracle.dgbtrs(A, ipiv, Bo, n, kl, ku, trans="T")
+    As = [torch.from_numpy(A[i].copy()).cuda() for i in range(batch)]
+    Ps = [torch.from_numpy(ipiv[i].copy()).cuda() for i in range(batch)]
+    Bs = [torch.from_numpy(B[i].copy()).cuda() for i in range(batch)]
+    bl.dgbtrs_batched("T", n, kl, ku, nrhs, bl.ptr_array(As), 2 * kl + ku + 1, bl.ptr_array(Ps),
+                      bl.ptr_array(Bs), n, batch)
+    torch.cuda.synchronize()
+    for i in range(batch):
+        assert np.all(same_bits(Bs[i].cpu().numpy(), Bo[i]))
+
+
 @pytest.mark.parametrize("batch,n,kl,ku", [(512, 193, 4, 4), (2000, 50, 10, 10)])
 def test_application_shaped_workloads(batch, n, kl, ku):
     """f4: XGC-like (512 x n=193) and PELE-like (n=50)

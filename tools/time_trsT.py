@@ -16,16 +16,17 @@ bl.dgbtrf_strided_batched(n, n, kl, ku, A, P, info)
 B0 = I.gen_rhs_torch(n, nrhs, count=batch, device="cuda")
 B = torch.empty_like(B0)
 b_trf, b_trs = I.alg_bytes(n, n, kl, ku, nrhs)
-for tr in ("N", "T"):
+for tr, var in (("N", bl.AUTO), ("T", bl.AUTO), ("T", bl.GENERIC)):
     ts = []
     for it in range(6):
         B.copy_(B0)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
-        bl.dgbtrs_strided_batched(tr, n, kl, ku, A, P, B)
+        bl.dgbtrs_strided_batched(tr, n, kl, ku, A, P, B, variant=var)
         e1.record()
         torch.cuda.synchronize()
         if it >= 2:
             ts.append(e0.elapsed_time(e1))
     ms = min(ts)
-    print(f"dgbtrs('{tr}') ({kl},{ku}) n={n} batch={batch} nrhs={nrhs}: {ms:.3f} ms, {batch * b_trs / ms / 1e6:.0f} GB/s")
+    vn = "generic" if var == bl.GENERIC else "auto"
+    print(f"dgbtrs('{tr}', {vn}) ({kl},{ku}) n={n} batch={batch} nrhs={nrhs}: {ms:.3f} ms, {batch * b_trs / ms / 1e6:.0f} GB/s")
