@@ -246,7 +246,7 @@ int bandlu_trs_rows_available(int kl, int ku);
  * returns their number L (0..2; < 0 on a negative argument) and, if kinds is
  * not NULL, writes L codes kinds[i] = 16 * kernel + bytes, kernel: 1 gbtrf_rows,
  * 2 gbtrf_window, 3 gbtrf_wide, 4 gbtrf_thread, 5 gbtrf_generic, 6 gbtrs_bwd,
- * 7 gbtrs_rows, 8 gbtrs_window, 9 gbtrs_generic, 10 gbtrf_thin; bytes (what the launch must
+ * 7 gbtrs_rows, 8 gbtrs_window, 9 gbtrs_generic, 10 gbtrf_thin, 11 gbtrs_blk; bytes (what the launch must
  * move per matrix): 1 factorization, 2 factorization + forward
  * substitution, 3 backward substitution, 4 full solve, 5 fused gbsv.
  * phase: 0, BANDLU_TRFS_TWO_LAUNCH, BANDLU_TRFS_FUSED or BANDLU_TRFS_THIN (as for dgbtrfs). */

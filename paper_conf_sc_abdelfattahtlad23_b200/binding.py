@@ -281,7 +281,7 @@ def trs_variant(n: int, kl: int, ku: int, nrhs: int) -> int:
 
 KERNEL_NAMES = {1: "gbtrf_rows_kernel", 2: "gbtrf_window_kernel", 3: "gbtrf_wide_kernel", 4: "gbtrf_thread_kernel",
                 5: "gbtrf_generic_kernel", 6: "gbtrs_bwd_kernel", 7: "gbtrs_rows_kernel", 8: "gbtrs_window_kernel",
-                9: "gbtrs_generic_kernel", 10: "gbtrf_thin_kernel"}
+                9: "gbtrs_generic_kernel", 10: "gbtrf_thin_kernel", 11: "gbtrs_blk_kernel"}
 BYTE_KINDS = {1: "trf", 2: "trf_fwd", 3: "trs_bwd", 4: "trs", 5: "gbsv"}
 TRFS_TWO_LAUNCH, TRFS_FUSED, TRFS_THIN = 16, 32, 64
 

@@ -24,6 +24,7 @@
 #include "gbtrs_bwd.cuh"
 #include "gbtrs_rows.cuh"
 #include "gbtrs_t.cuh"
+#include "gbtrs_blk.cuh"
 #include "gbtrs_window.cuh"
 #include "generic.cuh"
 #include "jit.cuh"
@@ -191,6 +192,16 @@ constexpr int64_t kTrsWarpsTarget = 148 * BANDLU_TRS_WPSM;
 #define BANDLU_TRST_WPSM BANDLU_TRS_WPSM
 #endif
 constexpr int64_t kTrsTWarpsTarget = 148 * BANDLU_TRST_WPSM;  // transposed solve (gbtrs_t.cuh)
+// ring solves: matrices per warp also bounded by shared memory, so that BANDLU_TRS_WPSM one-warp
+// CTAs still fit on an SM (a 32-matrix (32,32) ring is 142 KB: one warp per SM)
+constexpr size_t kTrsSmemPerWarp = 227 * 1024 / BANDLU_TRS_WPSM;
+template <class F>
+int trs_fit_gpw(int gpw, F smem_of) {
+#ifndef BANDLU_TRS_NO_FIT
+    while (gpw > 1 && smem_of(gpw) > kTrsSmemPerWarp) gpw >>= 1;
+#endif
+    return gpw;
+}
 
 inline int cuda_ret(cudaError_t e) { return e == cudaSuccess ? 0 : BANDLU_ERR_CUDA + (int)e; }
 
@@ -399,6 +410,21 @@ int jit_launch_trs_window(int kl, int ku, int n, int nrhs, Strided<const double>
     int R = nrhs >= 32 ? 32 : pow2_ceil(nrhs);
     int chunks = (nrhs + 31) / 32;
     const bool pairs = R >= 2;
+    if (nrhs == 1 && fwd) {  // the block-granular solve, as for compiled bands
+        const bandlu_jit::Kern &K = bandlu_jit::blk(kl, ku);
+        if (!K.ok) return BANDLU_ERR_UNSUPPORTED;
+        int gpw = 32;
+        while (gpw > 1 && (int64_t)batch < (int64_t)gpw * kTrsWarpsTarget) gpw >>= 1;
+        gpw = trs_fit_gpw(gpw, [&](int x) { return (size_t)(K.geo[0] + (long long)x * K.geo[1]) * 8; });
+        const size_t sm = (size_t)(K.geo[0] + (long long)gpw * K.geo[1]) * 8;
+        if (sm > 48 * 1024) {
+            cudaError_t e = cudaFuncSetAttribute((const void *)K.k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+            if (e != cudaSuccess) return cuda_ret(e);
+        }
+        const unsigned grid = (unsigned)((batch + gpw - 1) / gpw);
+        void *args[] = {&n, &nrhs, &A, &ldab, &P, &B, &ldb, &skip, &batch, &R, &chunks, &gpw, &fwd};
+        return cuda_ret(cudaLaunchKernel((const void *)K.k, dim3(grid), dim3(32), args, sm, st));
+    }
     const bandlu_jit::Kern &K = bandlu_jit::window(kl, ku, pairs);
     if (!K.ok) return BANDLU_ERR_UNSUPPORTED;
     const int64_t units = (int64_t)batch * chunks;
@@ -406,6 +432,7 @@ int jit_launch_trs_window(int kl, int ku, int n, int nrhs, Strided<const double>
     while (gpw > 1 && units < (int64_t)gpw * kTrsWarpsTarget) gpw >>= 1;
     int li = 0;
     while ((1 << li) < R) ++li;
+    gpw = trs_fit_gpw(gpw, [&](int x) { return (size_t)(K.geo[0] + (long long)x * K.geo[1 + li]) * 8; });
     const size_t sm = (size_t)(K.geo[0] + (long long)gpw * K.geo[1 + li]) * 8;
     if (sm > 48 * 1024) {
         cudaError_t e = cudaFuncSetAttribute((const void *)K.k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
@@ -524,9 +551,36 @@ int run_trf(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int b
 }
 
 // ------------------------------------------------------------------ trs
+// block-granular ring solve (gbtrs_blk.cuh), lane per (matrix, RHS column)
+template <int KL, int KU, class AP, class PP, class BP>
+int launch_trs_blk(int n, int nrhs, AP A, int ldab, PP P, BP B, int ldb, const int *skip, int batch,
+                   cudaStream_t st, int fwd = 1) {
+    using C = TrsBlk<KL, KU>;
+    const int R = nrhs >= 32 ? 32 : pow2_ceil(nrhs);
+    const int chunks = (nrhs + 31) / 32;
+    auto k = gbtrs_blk_kernel<KL, KU, AP, PP, BP>;
+    const int64_t units = (int64_t)batch * chunks;
+    int gpw = 32 / R;
+    while (gpw > 1 && units < (int64_t)gpw * kTrsWarpsTarget) gpw >>= 1;
+    gpw = trs_fit_gpw(gpw, [&](int x) { return C::smem_bytes(R, x); });
+    const size_t sm = C::smem_bytes(R, gpw);
+    if (int r = set_smem(k, sm)) return r;
+    const unsigned grid = (unsigned)((units + gpw - 1) / gpw);
+    k<<<grid, 32, sm, st>>>(n, nrhs, A, ldab, P, B, ldb, skip, batch, R, chunks, gpw, fwd);
+    return cuda_ret(cudaGetLastError());
+}
+
 template <int KL, int KU, class AP, class PP, class BP>
 int launch_trs_window(int n, int nrhs, AP A, int ldab, PP P, BP B, int ldb, const int *skip, int batch,
                       cudaStream_t st, int fwd = 1) {
+    // one RHS, full solve: the block-granular solve (C3 0.54 vs 0.61 ms, (32,32) n = 2048 5.3 vs
+    // 9.4 ms); nrhs >= 2 (C4 2.03 vs 2.10 ms) and the backward-only pass after a forward-fused
+    // factorization ((32,32) C5 points 1-4% faster) keep the row-pair window solve -- DESIGN.md Sec. 6
+#if defined(BANDLU_TRS_BLK_ALL)
+    return launch_trs_blk<KL, KU>(n, nrhs, A, ldab, P, B, ldb, skip, batch, st, fwd);
+#elif !defined(BANDLU_TRS_NO_BLK)
+    if (nrhs == 1 && fwd) return launch_trs_blk<KL, KU>(n, nrhs, A, ldab, P, B, ldb, skip, batch, st, fwd);
+#endif
     using C = TrsWin<KL, KU>;
     const int R = nrhs >= 32 ? 32 : pow2_ceil(nrhs);
     const int chunks = (nrhs + 31) / 32;
@@ -537,6 +591,7 @@ int launch_trs_window(int n, int nrhs, AP A, int ldab, PP P, BP B, int ldb, cons
     // SM (all four schedulers busy) before packing more of them into a warp.
     int gpw = 32 / R;
     while (gpw > 1 && units < (int64_t)gpw * kTrsWarpsTarget) gpw >>= 1;
+    gpw = trs_fit_gpw(gpw, [&](int x) { return C::smem_bytes(R, x, pairs); });
     const size_t sm = C::smem_bytes(R, gpw, pairs);
     if (int r = set_smem(k, sm)) return r;
     const unsigned grid = (unsigned)((units + gpw - 1) / gpw);
@@ -604,6 +659,7 @@ int launch_trs_t(int n, int nrhs, AP A, int ldab, PP P, BP B, int ldb, int batch
     const int64_t units = (int64_t)batch * chunks;
     int gpw = 32 / R;
     while (gpw > 1 && units < (int64_t)gpw * kTrsTWarpsTarget) gpw >>= 1;
+    gpw = trs_fit_gpw(gpw, [&](int x) { return C::smem_bytes(R, x); });
     const size_t sm = C::smem_bytes(R, gpw);
     if (int r = set_smem(k, sm)) return r;
     const unsigned grid = (unsigned)((units + gpw - 1) / gpw);
@@ -622,6 +678,7 @@ int jit_launch_trs_t(int kl, int ku, int n, int nrhs, Strided<const double> A, i
     while (gpw > 1 && units < (int64_t)gpw * kTrsTWarpsTarget) gpw >>= 1;
     int li = 0;
     while ((1 << li) < R) ++li;
+    gpw = trs_fit_gpw(gpw, [&](int x) { return (size_t)(K.geo[0] + (long long)x * K.geo[1 + li]) * 8; });
     const size_t sm = (size_t)(K.geo[0] + (long long)gpw * K.geo[1 + li]) * 8;
     if (sm > 48 * 1024) {
         cudaError_t e = cudaFuncSetAttribute((const void *)K.k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
@@ -713,6 +770,9 @@ int launch_trs_bwd(int n, AP A, int ldab, PP P, BP B, int ldb, int batch, cudaSt
         if (trs_rows_preferred(KL, KU)) return launch_trs_rows<KL, KU>(n, 1, A, ldab, P, B, ldb, nullptr, batch, st, 0);
     }
 #endif
+#ifdef BANDLU_TRS_BWD_BLK
+    return launch_trs_blk<KL, KU>(n, 1, A, ldab, P, B, ldb, nullptr, batch, st, 0);
+#endif
 #ifndef BANDLU_TRS_BWD_WINDOW
     if constexpr (std::is_same_v<AP, Strided<const double>> && KL + KU + 1 <= 32)
         return launch_trs_bwd_lean<KL, KU>(n, A, ldab, B, batch, st);
@@ -790,7 +850,7 @@ bool rows_ysm_fits_rt(int n, int kl, int ku) {
 
 // kernel ids / byte classes reported by bandlu_trfs_plan (include/bandlu.h)
 enum { KN_TRF_ROWS = 1, KN_TRF_WINDOW, KN_TRF_WIDE, KN_TRF_THREAD, KN_TRF_GENERIC, KN_TRS_BWD, KN_TRS_ROWS,
-       KN_TRS_WINDOW, KN_TRS_GENERIC, KN_TRF_THIN };
+       KN_TRS_WINDOW, KN_TRS_GENERIC, KN_TRF_THIN, KN_TRS_BLK };
 enum { KB_TRF = 1, KB_TRF_FWD, KB_TRS_BWD, KB_TRS, KB_GBSV };
 
 // run-time compiled bands, nrhs == 1: is the fused kernel picked?  (geometry from the
@@ -843,7 +903,8 @@ int trfs_plan(int n, int kl, int ku, int nrhs, int64_t batch, int phase, int *ki
     put(tv == BANDLU_ROWS ? (trf_wide_available(kl, ku) ? KN_TRF_WIDE : KN_TRF_ROWS)
         : tv == BANDLU_WINDOW ? KN_TRF_WINDOW : tv == BANDLU_THREAD ? KN_TRF_THREAD : KN_TRF_GENERIC, KB_TRF);
     const int sv = pick_trs(n, kl, ku, nrhs);
-    put(sv == BANDLU_ROWS ? KN_TRS_ROWS : sv == BANDLU_WINDOW ? KN_TRS_WINDOW : KN_TRS_GENERIC, KB_TRS);
+    put(sv == BANDLU_ROWS ? KN_TRS_ROWS : sv == BANDLU_WINDOW ? (nrhs == 1 ? KN_TRS_BLK : KN_TRS_WINDOW) : KN_TRS_GENERIC,
+        KB_TRS);
     return k;
 }
 

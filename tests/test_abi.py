@@ -152,11 +152,13 @@ def test_trfs_plan_reports_the_launches(lib):
     assert p["kernels"] == ["gbtrf_wide_kernel", "gbtrs_window_kernel"] and not p["fused"]
     p = b.trfs_plan(1024, 2, 32, 1, 100)  # kl+ku+1+PF > 2G: no fused kernel for (2,32)
     assert p["kernels"] == ["gbtrf_rows_kernel", "gbtrs_window_kernel"] and not p["fused"]
+    p = b.trfs_plan(512, 10, 10, 1, 1000, b.TRFS_TWO_LAUNCH)
+    assert p["kernels"] == ["gbtrf_rows_kernel", "gbtrs_bwd_kernel"]
     p = b.trfs_plan(1024, 2, 32, 16, 5000)
     assert p["kernels"] == ["gbtrf_rows_kernel", "gbtrs_window_kernel"] and p["bytes"] == ["trf", "trs"]
     p = b.trfs_plan(100, 5, 9, 1, 10, b.TRFS_TWO_LAUNCH)  # (5,9): not instantiated ahead of time
     if b.jit_band(5, 9):  # run-time compiled (NVRTC) kernels
-        assert p["kernels"][0] == "gbtrf_rows_kernel" and p["kernels"][1] in ("gbtrs_bwd_kernel", "gbtrs_window_kernel")
+        assert p["kernels"][0] == "gbtrf_rows_kernel" and p["kernels"][1] in ("gbtrs_bwd_kernel", "gbtrs_window_kernel", "gbtrs_blk_kernel")
     else:
         assert p["kernels"] == ["gbtrf_generic_kernel", "gbtrs_generic_kernel"]
     assert b.trfs_plan(0, 1, 1, 1, 10)["kernels"] == []

@@ -384,6 +384,42 @@ def test_trs_transposed_ring_kernel(kl, ku, n, nrhs, batch):
         assert np.all(same_bits(Bg.cpu().numpy(), Bo)), variant  # incl. the NaN padding row of ldb
 
 
+# block-granular one-RHS solve (gbtrs_blk.cuh; what dgbtrs / dgbsv run for nrhs == 1 on
+# window bands): n around kl and kv, odd and even ldab (the ring's 16-byte parity flips per
+# column) and ldb (the RHS pair phase), ragged batches that leave warps partly empty
+@pytest.mark.parametrize("kl,ku", [(10, 10), (2, 3), (32, 32), (2, 32), (10, 7), (5, 9)])
+@pytest.mark.parametrize("n,batch,ldab_extra,ldb_extra", [(1, 3, 0, 0), (4, 9, 1, 1), (11, 37, 0, 1),
+                                                          (21, 5, 1, 0), (66, 41, 1, 1), (300, 70, 0, 0)])
+def test_trs_blk_one_rhs(kl, ku, n, batch, ldab_extra, ldb_extra):
+    ldab = 2 * kl + ku + 1 + ldab_extra
+    A = I.gen_band(n, n, kl, ku, ldab=ldab, count=batch)
+    ipiv, info = oracle.dgbtrf(A, n, n, kl, ku)
+    B = I.gen_rhs(n, 1, ldb=n + ldb_extra, count=batch)
+    Bo = B.copy()
+    oracle.dgbtrs(A, ipiv, Bo, n, kl, ku)
+    Ag = torch.from_numpy(A).cuda(); Pg = torch.from_numpy(ipiv).cuda(); Bg = torch.from_numpy(B).cuda()
+    bl.dgbtrs_strided_batched("N", n, kl, ku, Ag, Pg, Bg, variant=bl.WINDOW)
+    torch.cuda.synchronize()
+    assert np.all(same_bits(Bg.cpu().numpy(), Bo))
+
+
+@pytest.mark.parametrize("kl,ku", [(10, 10), (2, 32), (32, 32), (5, 9)])
+@pytest.mark.parametrize("n,nrhs,batch", [(9, 1, 13), (70, 3, 21), (200, 1, 40)])
+def test_trs_transposed_odd_ldab_ldb(kl, ku, n, nrhs, batch):
+    """The transposed ring solve with an odd leading dimension (factor-range parity flips per
+    column) and odd ldb, bitwise vs the oracle."""
+    ldab = 2 * kl + ku + 2 + ((2 * kl + ku + 2) % 2 == 0)
+    A = I.gen_band(n, n, kl, ku, ldab=ldab, count=batch)
+    ipiv, info = oracle.dgbtrf(A, n, n, kl, ku)
+    B = I.gen_rhs(n, nrhs, ldb=n + 1 + (n % 2 == 0), count=batch)
+    Bo = B.copy()
+    oracle.dgbtrs(A, ipiv, Bo, n, kl, ku, trans="T")
+    Ag = torch.from_numpy(A).cuda(); Pg = torch.from_numpy(ipiv).cuda(); Bg = torch.from_numpy(B).cuda()
+    bl.dgbtrs_strided_batched("T", n, kl, ku, Ag, Pg, Bg, variant=bl.WINDOW)
+    torch.cuda.synchronize()
+    assert np.all(same_bits(Bg.cpu().numpy(), Bo))
+
+
 def test_trs_transposed_pointer_array():
     n, kl, ku, nrhs, batch = 60, 10, 10, 2, 11
     A = I.gen_band(n, n, kl, ku, count=batch)

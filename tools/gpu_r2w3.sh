@@ -1,0 +1,13 @@
+#!/bin/bash
+OUT=gpurun_out; mkdir -p $OUT
+timeout 900 python -m pytest tests/test_gpu_parity.py -q -x -k "trs or gbsv or trfs or fused or full or jit" > $OUT/pytest_w3.log 2>&1; echo "pytest rc=$? $(tail -1 $OUT/pytest_w3.log)"
+for a in "10 10 512 10000 1" "32 32 512 2000 1" "32 32 32 379356 1" "2 32 1024 5000 16"; do timeout 120 python tools/time_trsT.py $a; done
+timeout 900 python bench.py --config C5 --steps 5 --warmup 3 --no-cpu --fill 0.1 --parity-sample 64 > $OUT/bench_C5_w3.json 2> $OUT/bench_C5_w3.err; echo "C5 rc=$?"
+python - <<'PY'
+import json,sys
+d=json.loads(open('gpurun_out/bench_C5_w3.json').read().strip().splitlines()[-1])
+print(d['value'], d['roofline']['frac'], d['parity'])
+by={}
+for p in d['sweep']: by.setdefault((p['kl'],p['ku']),[]).append(p)
+for k,v in by.items(): print(k, 'ms=%.1f'%sum(p['ms_per_step'] for p in v), 'bwd ms', ' '.join('%.2f'%p['kernel_ms'][-1] for p in v))
+PY

@@ -16,7 +16,8 @@ OUT = os.path.join(ROOT, "gpurun_out")
 PROF = os.environ.get("PROF_DIR") or os.path.join(ROOT, "profiles")  # the GPU box writes into gpurun_out/
 
 KERNELS = ("gbtrf_tpm_kernel", "gbtrf_rows_kernel", "gbtrf_window_kernel", "gbtrf_wide_kernel", "gbtrf_tc_kernel", "gbtrf_generic_kernel",
-           "gbtrs_window_kernel", "gbtrs_bwd_kernel", "gbtrs_rows_kernel", "gbtrs_generic_kernel", "gbtrs_t_generic_kernel")
+           "gbtrs_window_kernel", "gbtrs_bwd_kernel", "gbtrs_rows_kernel", "gbtrs_generic_kernel", "gbtrs_t_generic_kernel",
+           "gbtrs_blk_kernel", "gbtrs_t_kernel")
 KEYS = {
     "duration_us": ("gpu__time_duration.sum", 1e-3),
     "dram_bytes_read": ("dram__bytes_read.sum", 1.0),
