@@ -145,7 +145,7 @@ class ClockSampler:
 # reference-arm timing and the post-timing parity check of a sample of the
 # GPU's outputs.  Neither is inside a timed GPU region.
 
-def cpu_oracle_rate(n, kl, ku, nrhs, seconds=6.0, sample=1024, threads=0):
+def cpu_oracle_rate(n, kl, ku, nrhs, seconds=6.0, sample=1024, threads=0, trans="N"):
     """The CPU oracle (OpenMP over the batch; threads=0: all host threads) on a
     bounded sample of the workload.  Returns a dict with matrices/s (best and
     median over the repetitions), the sample size, threads used and reps."""
@@ -163,16 +163,16 @@ def cpu_oracle_rate(n, kl, ku, nrhs, seconds=6.0, sample=1024, threads=0):
         A, B = A0.copy(), B0.copy()
         t0 = time.perf_counter()
         ipiv, info = oracle.dgbtrf(A, n, n, kl, ku, nthreads=threads)
-        oracle.dgbtrs(A, ipiv, B, n, kl, ku, nthreads=threads)
+        oracle.dgbtrs(A, ipiv, B, n, kl, ku, trans=trans, nthreads=threads)
         times.append(time.perf_counter() - t0)
     return {"best": sample / min(times), "median": sample / statistics.median(times), "sample": sample,
             "threads": used, "reps": len(times)}
 
 
-def cpu_baseline_entry(n, kl, ku, nrhs, flops_per_matrix, seconds=6.0):
-    allt = cpu_oracle_rate(n, kl, ku, nrhs, seconds=seconds)
+def cpu_baseline_entry(n, kl, ku, nrhs, flops_per_matrix, seconds=6.0, trans="N"):
+    allt = cpu_oracle_rate(n, kl, ku, nrhs, seconds=seconds, trans=trans)
     one = cpu_oracle_rate(n, kl, ku, nrhs, seconds=max(2.0, seconds / 3), sample=max(16, allt["sample"] // 8),
-                          threads=1)
+                          threads=1, trans=trans)
     g = lambda r: r * flops_per_matrix / 1e9  # noqa: E731
     return {"value": g(allt["best"]), "unit": "GFLOP/s", "cores": allt["threads"], "kind": "oracle",
             "matrices_per_s": allt["best"], "median_gflops": g(allt["median"]),
@@ -183,7 +183,7 @@ def cpu_baseline_entry(n, kl, ku, nrhs, flops_per_matrix, seconds=6.0):
                       f"{one['sample']} matrices on 1 thread (best of {one['reps']})"}
 
 
-def parity_check(idx_global, outs, n, kl, ku, nrhs):
+def parity_check(idx_global, outs, n, kl, ku, nrhs, trans="N"):
     """Bitwise comparison of GPU outputs (A, ipiv, B, info per sampled matrix)
     with the oracle recomputed from the same seeded inputs (runs of consecutive
     matrices regenerated and factored as one OpenMP batch).  Returns mismatches."""
@@ -201,7 +201,7 @@ def parity_check(idx_global, outs, n, kl, ku, nrhs):
         Ao = I.gen_band(n, n, kl, ku, count=cnt, first=idx[k])
         Bo = I.gen_rhs(n, nrhs, count=cnt, first=idx[k])
         ipo, info_o = oracle.dgbtrf(Ao, n, n, kl, ku)
-        oracle.dgbtrs(Ao, ipo, Bo, n, kl, ku)
+        oracle.dgbtrs(Ao, ipo, Bo, n, kl, ku, trans=trans)
         sl = slice(k, e + 1)
         ok = ((Ig[sl] == info_o) & np.all(Pg[sl] == ipo, axis=1) & same(Ag[sl], Ao) & same(Bg[sl], Bo))
         bad += int(np.sum(~ok))
@@ -257,6 +257,8 @@ def parse(argv=None):
     ap.add_argument("--plan", default="auto", choices=["auto", "two", "fused", "thin"],
                     help="dgbtrfs plan: the library's choice, the two-launch plan (factorization + forward, then "
                          "backward), or the fused single-launch kernel")
+    ap.add_argument("--trans", default="N", choices=["N", "T"],
+                    help="T: the step is dgbtrf then dgbtrs('T') (A^T X = B, SURVEY 8(f) f2), two launches")
     ap.add_argument("--c5-ns", default="", help="C5: comma-separated n list (default 32,64,128..2048 step 128)")
     args = ap.parse_args(argv)
     args.warmup = max(args.warmup, 3)
@@ -284,8 +286,13 @@ def run_config(args):
     f_trf, f_trs = I.nominal_flops(n, kl, ku, nrhs)
     xph = {"auto": 0, "two": bl.TRFS_TWO_LAUNCH, "fused": bl.TRFS_FUSED, "thin": bl.TRFS_THIN}[args.plan]
     plan = bl.trfs_plan(n, kl, ku, nrhs, cnt, xph)  # the kernels one dgbtrfs call launches
+    if args.trans == "T":  # dgbtrf (no forward fusion: nrhs 2 never fuses it) + dgbtrs('T')
+        plan = {"kernels": [bl.trfs_plan(n, kl, ku, 2, cnt, 0)["kernels"][0], "gbtrs_t_kernel"],
+                "bytes": ["trf", "trs"], "fused": False}
     per_launch_bytes = [I.alg_bytes_kind(n, kl, ku, nrhs, k) for k in plan["bytes"]]
     big = cnt * n * ldab * 8 > 2 * 126e6
+    if args.trans == "T":
+        desc += "; solve A^T X = B (dgbtrs 'T')"
     config = {"workload": desc, "global_batch": glob, "batch_per_gpu": cnt, "n": n, "kl": kl, "ku": ku,
               "nrhs": nrhs, "ldab": ldab, "layout": "strided LAPACK band (minimal ldab)",
               "parallelism": f"batch-shard x{world} ({args.scaling} scaling)",
@@ -309,6 +316,14 @@ def run_config(args):
         # (phase 1, phase 2 when there is a second one) are timed separately
         if evs is not None:
             evs[0].record(st)
+        if args.trans == "T":
+            bl.dgbtrf_strided_batched(n, n, kl, ku, A, P, info)
+            if evs is not None:
+                evs[1].record(st)
+            bl.dgbtrs_strided_batched("T", n, kl, ku, A, P, B)
+            if evs is not None:
+                evs[2].record(st)
+            return
         for ph in range(1, nph + 1):
             bl.dgbtrfs_strided_batched(n, kl, ku, A, P, B, info, phase=(ph if nph > 1 else 0) | xph)
             if evs is not None:
@@ -341,13 +356,13 @@ def run_config(args):
     sel = torch.tensor(loc, device=dev)
     outs = tuple(t.index_select(0, sel).cpu().numpy() for t in (A, P, B, info))
     ninfo = int((info != 0).sum())
-    bad = parity_check([lo + i for i in loc], outs, n, kl, ku, nrhs)
+    bad = parity_check([lo + i for i in loc], outs, n, kl, ku, nrhs, args.trans)
     summ = bd.gather_summaries([len(loc), bad, ninfo], dev)
     checked, mism, ninfo = (int(sum(s[k] for s in summ)) for k in range(3))
 
     # ---- e2e through the host-buffer C-ABI entry point (H2D + D2H timed)
     e2e = None
-    if args.e2e_steps > 0:
+    if args.e2e_steps > 0 and args.trans == "N":  # the host-buffer entry point is dgbsv ('N')
         Ah = A0.cpu().pin_memory()
         Bh = B0.cpu().pin_memory()
         Ahw, Bhw = torch.empty_like(Ah).pin_memory(), torch.empty_like(Bh).pin_memory()
@@ -409,7 +424,7 @@ def run_config(args):
         "clocks": clocks,
     }
     if world == 1 and not args.no_cpu:
-        line["cpu_baseline"] = cpu_baseline_entry(n, kl, ku, nrhs, f_trf + f_trs)
+        line["cpu_baseline"] = cpu_baseline_entry(n, kl, ku, nrhs, f_trf + f_trs, trans=args.trans)
     print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
@@ -535,8 +550,10 @@ def run_reference(args):
         bcfg = args.batch
     glob = bcfg * world if args.scaling == "weak" else bcfg
     f_trf, f_trs = I.nominal_flops(n, kl, ku, nrhs)
-    r = cpu_oracle_rate(n, kl, ku, nrhs, seconds=max(3.0, 0.5 * args.steps))
+    r = cpu_oracle_rate(n, kl, ku, nrhs, seconds=max(3.0, 0.5 * args.steps), trans=args.trans)
     gflops = r["best"] * (f_trf + f_trs) / 1e9
+    if args.trans == "T":
+        desc += "; solve A^T X = B (dgbtrs 'T')"
     config = {"workload": desc, "global_batch": glob, "n": n, "kl": kl, "ku": ku, "nrhs": nrhs,
               "ldab": 2 * kl + ku + 1, "parallelism": f"batch-shard x{world} ({args.scaling} scaling)"}
     line = {"impl": "reference", "metric": METRIC, "value": gflops, "unit": "GFLOP/s", "n_gpus": world,

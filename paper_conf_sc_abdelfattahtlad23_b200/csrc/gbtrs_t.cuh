@@ -25,6 +25,8 @@
 //    and division (the order of every chain is unchanged).  Measured C3
 //    (10,10), n = 512, 10^4 matrices: 0.616 ms vs 0.915 ms with a wait and
 //    barrier per step, vs 3.46 ms for the thread-per-column generic kernel.
+//  * Each lane copies the RHS rows of a block as 16-byte aligned pairs (not one
+//    8-byte copy per row: at 16 RHS per matrix that was the LSU cost).
 //  * The first kv steps of pass 1 and the last kl steps of pass 2 (the
 //    truncated dot products) run straight from global memory, so the ring
 //    loop has no per-element predicates.
@@ -53,14 +55,16 @@ struct TrsT {
     static constexpr int NB1 = (STEPS + UB1 - 1) / UB1 < 2 ? 2 : (STEPS + UB1 - 1) / UB1;
     static constexpr int NB2 = (STEPS + UB2 - 1) / UB2 < 2 ? 2 : (STEPS + UB2 - 1) / UB2;
     static constexpr int NS1 = NB1 * UB1, NS2 = NB2 * UB2;  // ring slots per pass
-    // pass-1 slot: [SP1: U rows 0..kv, 16-byte rounded][R rhs]; pass-2 slot: [SP2: L rows][ipiv, pad][R rhs]
+    // pass-1 slot: [SP1: U rows 0..kv, 16-byte rounded]; pass-2 slot: [SP2: L rows][ipiv, pad].
+    // RHS rows move per block: each lane copies the UB rows a block consumes as 16-byte aligned
+    // pairs (UB + 2 doubles at most) into its area of the block's RHS buffer.
     static constexpr int SP1 = ((KV + 1 + 2) + 1) & ~1;
     static constexpr int SP2 = ((KL + 2) + 1) & ~1;
-    __host__ __device__ static constexpr int slot1(int R) { return SP1 + ((R + 1) & ~1); }
-    __host__ __device__ static constexpr int slot2(int R) { return SP2 + 2 + ((R + 1) & ~1); }
-    __host__ __device__ static constexpr int ring_dbl(int R) {
-        return NS1 * slot1(R) > NS2 * slot2(R) ? NS1 * slot1(R) : NS2 * slot2(R);
-    }
+    static constexpr int SL1 = SP1, SL2 = SP2 + 2;
+    static constexpr int RB1 = ((UB1 + 2) + 1) & ~1, RB2 = ((UB2 + 2) + 1) & ~1;
+    __host__ __device__ static constexpr int p1_dbl(int R) { return NS1 * SL1 + NB1 * RB1 * R; }
+    __host__ __device__ static constexpr int p2_dbl(int R) { return NS2 * SL2 + NB2 * RB2 * R; }
+    __host__ __device__ static constexpr int ring_dbl(int R) { return p1_dbl(R) > p2_dbl(R) ? p1_dbl(R) : p2_dbl(R); }
     // pitch == 2 (mod 4) doubles: the groups' reads of one slot offset sit in different banks
     __host__ __device__ static constexpr int group_dbl(int R) { return ring_dbl(R) + (6 - ring_dbl(R) % 4) % 4; }
     static constexpr int PAD = 2;
@@ -84,16 +88,32 @@ __global__ void __launch_bounds__(32)
     const bool act = live && (r0 + t < nrhs);  // lane solves (and stores) a column
     if (__ballot_sync(0xffffffffu, live) == 0u) return;
 
-    const int GD = C::group_dbl(R), SD1 = C::slot1(R), SD2 = C::slot2(R);
+    const int GD = C::group_dbl(R);
+    constexpr int SD1 = C::SL1, SD2 = C::SL2, RB1 = C::RB1, RB2 = C::RB2;
     double *gring = smem + C::PAD + (g < gpw ? g : 0) * GD;
     const double *ab = live ? A.get(mat) : nullptr;
     const int *ipiv = live ? P.get(mat) : nullptr;
     double *bcol = act ? B.get(mat) + (int64_t)(r0 + t) * ldb : nullptr;
     const void *dummy = g_dummy;
     const uint32_t gring_s = smem_u32(gring);
-    auto issue_row = [&](uint32_t dst, int q) {  // this lane's RHS row q
+    // this lane's RHS rows qlo..qlo+cnt-1 (zero outside 0..n-1) -> dst as 16-byte aligned pairs
+    // starting at row qlo - o, o = (qlo + ph) & 1
+    const int ph = act ? (int)((reinterpret_cast<uintptr_t>(bcol) >> 3) & 1) : 0;
+    auto issue_rows = [&](uint32_t dst, int qlo, int cnt) {
         if (g >= gpw) return;
-        cp_async8(dst, act ? (const void *)(bcol + q) : dummy, act ? 8u : 0u);
+        const int q0 = qlo - ((qlo + ph) & 1);
+        for (int r = q0; r < qlo + cnt; r += 2, dst += 16) {
+            if (act && r >= 0 && r + 1 < n) {
+                cp_async16(dst, bcol + r, 16u);
+            } else if (act && r >= 0 && r < n) {  // last row: its 8 bytes, zero-fill the rest
+                cp_async16(dst, bcol + r, 8u);
+            } else if (act && r == -1 && n > 0) {  // (row -1, row 0)
+                st_shared_f64_if(true, dst, 0.0);
+                cp_async8(dst + 8, bcol, 8u);
+            } else {
+                cp_async16(dst, dummy, 0u);
+            }
+        }
     };
     // parity of a factor range's first element: its offset inside the 16-byte aligned slot
     auto delta_of = [&](int64_t lo) { return live ? (int)((reinterpret_cast<uintptr_t>(ab + lo) >> 3) & 1) : 0; };
@@ -127,14 +147,19 @@ __global__ void __launch_bounds__(32)
     }
     const int n1 = n - KV;  // steps k = 0..n1-1: column j = KV + k, U rows 0..KV (slot k % NS1)
     if (n1 > 0) {
+        // block b: steps b*UB1 .. +UB1-1 and their rows b(KV + k) (RHS buffer b % NB1)
+        const uint32_t rhs1 = gring_s + (uint32_t)((NS1 * SD1 + t * RB1) * 8);
         auto issue_blk = [&](int b) {  // the UB1 steps of block b, one cp.async group
+            if (b * UB1 < n1) {
+                if (clive) {
 #pragma unroll 1
-            for (int s = 0; s < UB1; ++s) {
-                const int k = b * UB1 + s;
-                if (k >= n1) break;
-                const int rs = k % NS1;
-                if (clive) issue_fac(cring_s + (uint32_t)(rs * SD1 * 8), (int64_t)(KV + k) * ldab, KV + 1);
-                issue_row(gring_s + (uint32_t)((rs * SD1 + C::SP1 + t) * 8), KV + k);
+                    for (int s = 0; s < UB1; ++s) {
+                        const int k = b * UB1 + s;
+                        if (k >= n1) break;
+                        issue_fac(cring_s + (uint32_t)((k % NS1) * SD1 * 8), (int64_t)(KV + k) * ldab, KV + 1);
+                    }
+                }
+                issue_rows(rhs1 + (uint32_t)((b % NB1) * R * RB1 * 8), KV + b * UB1, UB1);
             }
             cp_async_commit();
         };
@@ -151,12 +176,13 @@ __global__ void __launch_bounds__(32)
             cp_async_wait<NB1 - 1>();
             __syncwarp();
             // no barrier inside the block: step s+1's dot product overlaps step s's division
+            const double *rin = gring + NS1 * SD1 + ((b % NB1) * R + t) * RB1 + ((KV + k0 + ph) & 1);
 #pragma unroll
             for (int s = 0; s < UB1; ++s) {
                 const int k = k0 + s, rs = k % NS1;
                 const double *slot = gring + rs * SD1;
                 const double *uc = slot + (d1 ^ ((k & 1) & dstep));  // uc[r] = AB(r, j) = U(j-KV+r, j)
-                double temp = slot[C::SP1 + t];                     // b(j)
+                double temp = rin[s];                               // b(j)
 #pragma unroll
                 for (int i = 0; i < KV; ++i) temp = __fma_rn(-uc[i], x[s + i], temp);
                 const double z = __ddiv_rn(temp, uc[KV]);  // steps past n1: stale slot, never stored
@@ -198,20 +224,21 @@ __global__ void __launch_bounds__(32)
             __syncwarp();
             // blocks of UB2 rows aligned to row 0: block bi covers rows bi*UB2 .. bi*UB2+UB2-1
             // (top block: rows > jb0 were done above); row j uses slot j % NS2
+            // (RHS buffer bi % NB2 holds rows bi*UB2 .. +UB2-1: z(j) for j <= jb0)
+            const uint32_t rhs2 = gring_s + (uint32_t)((NS2 * SD2 + t * RB2) * 8);
             auto issue_blk = [&](int bi) {
                 if (bi >= 0) {
+                    if (clive) {
 #pragma unroll 1
-                    for (int p = UB2 - 1; p >= 0; --p) {
-                        const int j = bi * UB2 + p;
-                        if (j > jb0) continue;
-                        const int rs = j % NS2;
-                        const uint32_t dst = cring_s + (uint32_t)(rs * SD2 * 8);
-                        if (clive) {
+                        for (int p = UB2 - 1; p >= 0; --p) {
+                            const int j = bi * UB2 + p;
+                            if (j > jb0) continue;
+                            const uint32_t dst = cring_s + (uint32_t)((j % NS2) * SD2 * 8);
                             if (cq == 0) cp_async4(dst + C::SP2 * 8, cipiv + j, 4u);
                             issue_fac(dst, (int64_t)j * ldab + KV + 1, KL);
                         }
-                        issue_row(gring_s + (uint32_t)((rs * SD2 + C::SP2 + 2 + t) * 8), j);
                     }
+                    issue_rows(rhs2 + (uint32_t)((bi % NB2) * R * RB2 * 8), bi * UB2, UB2);
                 }
                 cp_async_commit();
             };
@@ -231,6 +258,7 @@ __global__ void __launch_bounds__(32)
             for (int bi = btop; bi >= 0; --bi) {
                 cp_async_wait<NB2 - 1>();
                 __syncwarp();
+                const double *rin = gring + NS2 * SD2 + ((bi % NB2) * R + t) * RB2 + ((bi * UB2 + ph) & 1);
 #pragma unroll
                 for (int s = 0; s < UB2; ++s) {
                     const int pj = UB2 - 1 - s;  // row j = bi*UB2 + pj
@@ -241,7 +269,7 @@ __global__ void __launch_bounds__(32)
                     double temp = 0.0;
 #pragma unroll
                     for (int i = 1; i <= KL; ++i) temp = __fma_rn(v[pj + i], lc[i - 1], temp);
-                    const double xj = run ? __dsub_rn(slot[C::SP2 + 2 + t], temp) : v[pj];
+                    const double xj = run ? __dsub_rn(rin[pj], temp) : v[pj];
                     const int d = run ? reinterpret_cast<const int *>(slot + C::SP2)[0] - 1 - j : 0;
                     double y = xj;  // interchange x(j) <-> x(j+d)
 #pragma unroll

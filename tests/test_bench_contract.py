@@ -93,3 +93,10 @@ def test_bench_parity_checker_catches_a_flipped_bit():
     assert bench.parity_check(loc, (A, ip, B, inf), n, kl, ku, 1) == 0
     A[3, 5, 5] = np.nextafter(A[3, 5, 5], np.inf)
     assert bench.parity_check(loc, (A, ip, B, inf), n, kl, ku, 1) == 1
+    # --trans T: the checker solves A^T X = B with the oracle
+    A = np.concatenate([I.gen_band(n, n, kl, ku, count=1, first=i) for i in loc])
+    B = np.concatenate([I.gen_rhs(n, 1, count=1, first=i) for i in loc])
+    ip, inf = oracle.dgbtrf(A, n, n, kl, ku)
+    oracle.dgbtrs(A, ip, B, n, kl, ku, trans="T")
+    assert bench.parity_check(loc, (A, ip, B, inf), n, kl, ku, 1, "T") == 0
+    assert bench.parity_check(loc, (A, ip, B, inf), n, kl, ku, 1, "N") == len(loc)
