@@ -24,15 +24,18 @@ struct TrfWide {
     static constexpr int KL = KL_, KU = KU_, KV = KL + KU, W = KV + 1;
     static constexpr int G = 64;                 // lanes per matrix (= the CTA)
 #ifndef BANDLU_WIDE_U
-#define BANDLU_WIDE_U 4
+#define BANDLU_WIDE_U 8
 #endif
-    static constexpr int U = BANDLU_WIDE_U;
+    // columns per block (preload / record / window-shift granularity): 8 measured 7% faster than 4
+    // on (32,32) (C5 724 vs 767 ms: the 138-register window shifts half as often); 4 where the
+    // KL+1 active rows + U preloaded rows would not fit the 64 lanes
+    static constexpr int U = (KL + 1 + BANDLU_WIDE_U <= G) ? BANDLU_WIDE_U : 4;
     static constexpr int WS = W + U, H = (WS + 1) / 2;
     static_assert(KL + 1 + U <= G, "slots");
     static constexpr int WPB = 2 * H + 4;
     static constexpr int WP = (WPB + 11) / 16 * 16 + 4;  // == 4 (mod 16) doubles
     static constexpr int RP = WP - 2;
-    static constexpr int D = 4, DB = D / U;
+    static constexpr int D = U > 4 ? U : 4, DB = D / U;  // staging lead (rows / blocks)
     static constexpr int RR = pow2_ceil((DB + 1) * U);
 #ifdef BANDLU_WIDE_ONESYNC
     static constexpr int NREC = 2 * U;  // one candidate record per warp and step (one barrier per step)
@@ -202,11 +205,17 @@ __global__ void __launch_bounds__(64, 4)
             const bool w1 = c1.w && (!c0.w || c1.x > c0.x || (c1.x == c0.x && (c1.y > c0.y || (c1.y == c0.y && c1.z < c0.z))));
             const bool is_piv = (w == (w1 ? 1 : 0)) && (lane == wl);
 
-            // ---- pivot row (U row j: slots s..s+KV) + (B entry, logical row) -> record s
+            // ---- pivot row (U row j: slots s..s+KV) + (B entry, logical row) -> record s; only the
+            // pivot's warp issues the stores (warp-uniform branch: the other warp skips KV/2 stores)
             const uint32_t rcs = rec_s + (uint32_t)(s * WP * 8);
+#ifndef BANDLU_WIDE_STORE_ALL
+            if (__any_sync(0xffffffffu, is_piv))
+#endif
+            {
 #pragma unroll
-            for (int h = s / 2; h <= (s + KV) / 2; ++h) st_shared_v2_if(is_piv, rcs + h * 16, v[h]);
-            st_shared_v2_if(is_piv, rcs + RP * 8, make_double2(bq, __longlong_as_double((long long)pos)));
+                for (int h = s / 2; h <= (s + KV) / 2; ++h) st_shared_v2_if(is_piv, rcs + h * 16, v[h]);
+                st_shared_v2_if(is_piv, rcs + RP * 8, make_double2(bq, __longlong_as_double((long long)pos)));
+            }
             __syncthreads();
 #endif
             const double2 yp = ld_shared_v2(rcs + RP * 8);

@@ -85,6 +85,22 @@ for kl, ku in BANDS:
     torch.cuda.synchronize()
     check(f"trsT {kl},{ku}", same(Bg.cpu().numpy(), Btt))
 
+# ring solves past the truncated edges (n > kv): 'N' one RHS (block solve) and 'T', nrhs 1 and 5
+for kl, ku in ((10, 10), (2, 32), (32, 32)):
+    n, batch = 150, 7
+    A0 = I.gen_band(n, n, kl, ku, count=batch)
+    Ao = A0.copy()
+    ipo, info_o = oracle.dgbtrf(Ao, n, n, kl, ku)
+    for nrhs in (1, 5):
+        B0 = I.gen_rhs(n, nrhs, ldb=n + 1, count=batch)
+        for tr in ("N", "T"):
+            Bt = B0.copy()
+            oracle.dgbtrs(Ao.copy(), ipo, Bt, n, kl, ku, trans=tr)
+            Bg = torch.from_numpy(B0.copy()).cuda()
+            bl.dgbtrs_strided_batched(tr, n, kl, ku, torch.from_numpy(Ao).cuda(), torch.from_numpy(ipo).cuda(), Bg)
+            torch.cuda.synchronize()
+            check(f"trs{tr} {kl},{ku} n{n} nrhs{nrhs}", same(Bg.cpu().numpy(), Bt))
+
 # pointer arrays, nrhs 3 (window solve), and the host path
 n, kl, ku, nrhs, batch = 33, 10, 10, 3, 9
 A0 = I.gen_band(n, n, kl, ku, count=batch)
