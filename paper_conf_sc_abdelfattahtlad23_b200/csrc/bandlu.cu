@@ -1131,6 +1131,9 @@ int bandlu_jit_check(int kl, int ku, char *log, int loglen) {
     }
     if (kl + ku + 1 <= 32) specs.push_back(bandlu_jit::bwd_spec(kl, ku, 8));
     specs.push_back(bandlu_jit::window_spec(kl, ku, true));
+    specs.push_back(bandlu_jit::window_spec(kl, ku, false));
+    specs.push_back(bandlu_jit::blk_spec(kl, ku));
+    specs.push_back(bandlu_jit::trst_spec(kl, ku));
     for (const auto &sp : specs) {
         std::vector<char> bin;
         std::string low;

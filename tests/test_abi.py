@@ -173,7 +173,7 @@ def test_jit_bands_compile_without_gpu(lib):
     from paper_conf_sc_abdelfattahtlad23_b200 import binding as b
     if not b.jit_band(5, 6):
         pytest.skip("NVRTC not available")
-    for kl, ku in [(5, 6), (16, 16), (0, 40), (33, 20)]:
+    for kl, ku in [(5, 6), (16, 16), (0, 40), (33, 20), (56, 4)]:  # (56, 4): wide, 4-column blocks
         assert b.jit_band(kl, ku)
         assert b.jit_check(kl, ku) == "", (kl, ku)
     assert not b.jit_band(10, 10) and not b.jit_band(2, 32)  # instantiated ahead of time
