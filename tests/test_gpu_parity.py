@@ -598,7 +598,7 @@ def test_fused_dgbsv_leaves_b_untouched_where_singular(kl, ku, n):
 # Bands no list instantiates ahead of time run the same templates compiled with
 # NVRTC on first use (jit.cuh; Sec. 8.1): every entry point and
 # plan must still equal the oracle bitwise.
-JIT_BANDS = [(5, 6), (16, 16), (20, 20), (0, 32), (7, 1), (33, 20)]
+JIT_BANDS = [(5, 6), (16, 16), (20, 20), (0, 32), (7, 1), (33, 20), (56, 4)]
 
 
 @pytest.mark.parametrize("kl,ku", JIT_BANDS)
