@@ -103,7 +103,11 @@ enum bandlu_variant {
                            update per panel (bandlu_tpm_available); bitwise equal results */
     BANDLU_THIN = 7     /* dgbtrf only, square, strided: thin bands, one thread per matrix with the
                            window in registers and whole band columns staged cooperatively through
-                           shared memory (bandlu_thin_available); bitwise equal results */
+                           shared memory (bandlu_thin_available); bitwise equal results */,
+    BANDLU_COLS = 8     /* dgbtrf (and dgbtrfs' factorization), square: thin lower bands (kl <= 4),
+                           the lanes of a group own the window's columns (gbtrf_cols.cuh);
+                           compiled (kl, ku) only (bandlu_cols_available); AUTO's choice where
+                           compiled.  Bitwise equal results */
 };
 
 /* ---- dgbtrf: band LU with partial pivoting ---- */
@@ -224,6 +228,8 @@ int bandlu_rows_available(int kl, int ku);
 int bandlu_thread_available(int kl, int ku);
 /* 1 if a thread-per-matrix shared-memory-window kernel (BANDLU_TPM) is compiled for (kl, ku), else 0. */
 int bandlu_tpm_available(int kl, int ku);
+/* 1 if a column-owner (BANDLU_COLS) factorization kernel is compiled for (kl, ku), else 0. */
+int bandlu_cols_available(int kl, int ku);
 /* 1 if a thin-band thread-per-matrix kernel (BANDLU_THIN) is compiled for (kl, ku), else 0
  * (only in -DBANDLU_WITH_THIN builds: measured slower, AUTO never picks it). */
 int bandlu_thin_available(int kl, int ku);

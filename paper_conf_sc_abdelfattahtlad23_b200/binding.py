@@ -18,7 +18,7 @@ import torch
 
 from . import _build
 
-AUTO, GENERIC, WINDOW, TC, ROWS, THREAD, TPM, THIN = 0, 1, 2, 3, 4, 5, 6, 7
+AUTO, GENERIC, WINDOW, TC, ROWS, THREAD, TPM, THIN, COLS = 0, 1, 2, 3, 4, 5, 6, 7, 8
 ERR_UNSUPPORTED, ERR_CUDA = 1000, 2000
 
 _lib = None
@@ -73,6 +73,7 @@ def load(build_if_missing: bool = False):
         "bandlu_thread_available": [i, i],
         "bandlu_tpm_available": [i, i],
         "bandlu_thin_available": [i, i],
+        "bandlu_cols_available": [i, i],
         "bandlu_jit_band": [i, i],
         "bandlu_jit_check": [i, i, p, i],
         "bandlu_trs_variant": [i, i, i, i],
@@ -91,7 +92,7 @@ def load(build_if_missing: bool = False):
 EXPORTS = ("dgbtrf_batched", "dgbtrf_strided_batched", "dgbtrf_strided_batched_ex", "dgbtrs_batched",
            "dgbtrs_strided_batched", "dgbtrs_strided_batched_ex", "dgbsv_batched", "dgbsv_strided_batched",
            "dgbsv_strided_batched_host", "dgbtrfs_strided_batched", "dgbtrfs_strided_batched_ex", "bandlu_trf_variant", "bandlu_trs_variant", "bandlu_tc_available", "bandlu_rows_available", "bandlu_trs_rows_available", "bandlu_thread_available",
-           "bandlu_tpm_available", "bandlu_thin_available", "bandlu_jit_band", "bandlu_jit_check", "bandlu_trfs_plan", "bandlu_version")
+           "bandlu_tpm_available", "bandlu_thin_available", "bandlu_cols_available", "bandlu_jit_band", "bandlu_jit_check", "bandlu_trfs_plan", "bandlu_version")
 
 
 def _stream(stream):
@@ -270,6 +271,11 @@ def jit_check(kl: int, ku: int) -> str:
     return "" if rc == 0 else buf.value.decode(errors="replace") or "failed"
 
 
+def cols_available(kl: int, ku: int) -> bool:
+    """True if a column-owner factorization kernel (dgbtrf variant COLS) is compiled for (kl, ku)."""
+    return bool(load().bandlu_cols_available(kl, ku))
+
+
 def trs_rows_available(kl: int, ku: int) -> bool:
     """True if a lane-per-row solve kernel (dgbtrs variant ROWS) is compiled for (kl, ku)."""
     return bool(load().bandlu_trs_rows_available(kl, ku))
@@ -281,7 +287,8 @@ def trs_variant(n: int, kl: int, ku: int, nrhs: int) -> int:
 
 KERNEL_NAMES = {1: "gbtrf_rows_kernel", 2: "gbtrf_window_kernel", 3: "gbtrf_wide_kernel", 4: "gbtrf_thread_kernel",
                 5: "gbtrf_generic_kernel", 6: "gbtrs_bwd_kernel", 7: "gbtrs_rows_kernel", 8: "gbtrs_window_kernel",
-                9: "gbtrs_generic_kernel", 10: "gbtrf_thin_kernel", 11: "gbtrs_blk_kernel"}
+                9: "gbtrs_generic_kernel", 10: "gbtrf_thin_kernel", 11: "gbtrs_blk_kernel",
+                12: "gbtrf_cols_kernel"}
 BYTE_KINDS = {1: "trf", 2: "trf_fwd", 3: "trs_bwd", 4: "trs", 5: "gbsv"}
 TRFS_TWO_LAUNCH, TRFS_FUSED, TRFS_THIN = 16, 32, 64
 

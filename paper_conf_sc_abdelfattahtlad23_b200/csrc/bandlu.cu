@@ -27,6 +27,7 @@
 #include "gbtrs_blk.cuh"
 #include "gbtrs_window.cuh"
 #include "generic.cuh"
+#include "gbtrf_cols.cuh"
 #include "jit.cuh"
 
 using namespace bandlu;
@@ -93,6 +94,31 @@ namespace {
     X(10, 7, 16, 1)                                      \
     X(2, 32, 8, 1)                                       \
     BANDLU_ROWS_THIN_LIST(X)
+#endif
+
+// (KL, KU, GL, CPL) compiled as column-owner kernels (gbtrf_cols.cuh; kl <= 4, square): GL lanes
+// per matrix with CPL column slots each (GL*CPL >= kl+ku+1); AUTO's choice where compiled.
+#if defined(BANDLU_NO_COLS)
+#define BANDLU_COLS_LIST(X)
+#elif defined(BANDLU_ONLY_C3)
+#define BANDLU_COLS_LIST(X) X(1, 1, 4, 1)
+#else
+#define BANDLU_COLS_LIST(X) \
+    X(0, 0, 4, 1)           \
+    X(0, 3, 4, 1)           \
+    X(1, 1, 4, 1)           \
+    X(2, 2, 4, 2)           \
+    X(2, 3, 4, 2)           \
+    X(3, 0, 4, 1)           \
+    X(3, 2, 4, 2)           \
+    BANDLU_COLS_EXTRA(X)
+#endif
+// opt-in (measured): (4,4) slower than the row-slot kernel (XGC-like 0.096 vs
+// 0.072 ms); (2,32) with 8 lanes x 5 slots no faster (1.60 vs 1.62 ms at C4)
+#ifdef BANDLU_COLS_WIDE
+#define BANDLU_COLS_EXTRA(X) X(4, 4, 4, 3) X(2, 32, 8, 5)
+#else
+#define BANDLU_COLS_EXTRA(X)
 #endif
 
 // (KL, KU, MPW) compiled as thread-per-matrix shared-memory-window kernels with rank-4
@@ -239,6 +265,18 @@ int launch_trf_rows(int m, int n, AP A, int ldab, PP P, int *info, int batch, cu
     return cuda_ret(cudaGetLastError());
 }
 
+template <int KL, int KU, int GL, int CPL, int FL, class AP, class PP, class BP>
+int launch_trf_cols(int n, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st, BP B) {
+    using C = TrfCols<KL, KU, GL, CPL>;
+    auto k = gbtrf_cols_kernel<KL, KU, GL, CPL, FL, AP, PP, BP>;
+    const size_t sm = C::smem_bytes();
+    if (int r = set_smem(k, sm)) return r;
+    const int64_t per_block = (int64_t)C::WARPS * C::GPW;
+    const unsigned grid = (unsigned)((batch + per_block - 1) / per_block);
+    k<<<grid, C::WARPS * 32, sm, st>>>(n, A, ldab, P, info, batch, B);
+    return cuda_ret(cudaGetLastError());
+}
+
 template <int KL, int KU, bool FWD, class AP, class PP, class BP>
 int launch_trf_wide(int m, int n, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st, BP B) {
     using C = TrfWide<KL, KU>;
@@ -327,6 +365,14 @@ bool trf_rows_available(int kl, int ku) {
     BANDLU_ROWS_LIST(X)
 #undef X
     return trf_wide_available(kl, ku);
+}
+
+bool trf_cols_available(int kl, int ku) {
+#define X(a, b, g, c) \
+    if (kl == a && ku == b) return true;
+    BANDLU_COLS_LIST(X)
+#undef X
+    return false;
 }
 
 bool trs_window_available(int kl, int ku) {
@@ -463,6 +509,7 @@ int jit_launch_trs_bwd(int kl, int ku, int n, Strided<const double> A, int ldab,
 int pick_trf(int m, int n, int kl, int ku) {
     if (m <= 0 || n <= 0) return BANDLU_GENERIC;
     if (jit_band(kl, ku)) return BANDLU_ROWS;  // compiled on first use (jit.cuh)
+    if (m == n && trf_cols_available(kl, ku)) return BANDLU_COLS;
     // BANDLU_TC is opt-in: measured slower than the row-owner window at C3
     // (1.54 vs 1.10 ms), so AUTO never picks it.
     if (trf_thread_preferred(kl, ku)) return BANDLU_THREAD;
@@ -489,6 +536,14 @@ int run_trf(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int b
 #define X(a, b) \
     if (kl == a && ku == b) return launch_trf_tc<a, b, false>(m, n, A, ldab, P, info, batch, st, Strided<double>{nullptr, 0});
         BANDLU_TC_LIST(X)
+#undef X
+        return BANDLU_ERR_UNSUPPORTED;
+    }
+    if (variant == BANDLU_COLS && m > 0 && n > 0) {
+        if (m != n) return BANDLU_ERR_UNSUPPORTED;
+#define X(a, b, g, c) \
+    if (kl == a && ku == b) return launch_trf_cols<a, b, g, c, 0>(n, A, ldab, P, info, batch, st, Strided<double>{nullptr, 0});
+        BANDLU_COLS_LIST(X)
 #undef X
         return BANDLU_ERR_UNSUPPORTED;
     }
@@ -545,7 +600,7 @@ int run_trf(int m, int n, int kl, int ku, AP A, int ldab, PP P, int *info, int b
         return BANDLU_ERR_UNSUPPORTED;
     }
     if (variant != BANDLU_GENERIC && variant != BANDLU_WINDOW && variant != BANDLU_TC && variant != BANDLU_ROWS &&
-        variant != BANDLU_THREAD && variant != BANDLU_TPM && variant != BANDLU_THIN)
+        variant != BANDLU_THREAD && variant != BANDLU_TPM && variant != BANDLU_THIN && variant != BANDLU_COLS)
         return BANDLU_ERR_UNSUPPORTED;
     return launch_trf_generic(m, n, kl, ku, A, ldab, P, info, batch, st);
 }
@@ -850,7 +905,7 @@ bool rows_ysm_fits_rt(int n, int kl, int ku) {
 
 // kernel ids / byte classes reported by bandlu_trfs_plan (include/bandlu.h)
 enum { KN_TRF_ROWS = 1, KN_TRF_WINDOW, KN_TRF_WIDE, KN_TRF_THREAD, KN_TRF_GENERIC, KN_TRS_BWD, KN_TRS_ROWS,
-       KN_TRS_WINDOW, KN_TRS_GENERIC, KN_TRF_THIN, KN_TRS_BLK };
+       KN_TRS_WINDOW, KN_TRS_GENERIC, KN_TRF_THIN, KN_TRS_BLK, KN_TRF_COLS };
 enum { KB_TRF = 1, KB_TRF_FWD, KB_TRS_BWD, KB_TRS, KB_GBSV };
 
 // run-time compiled bands, nrhs == 1: is the fused kernel picked?  (geometry from the
@@ -890,6 +945,12 @@ int trfs_plan(int n, int kl, int ku, int nrhs, int64_t batch, int phase, int *ki
         put(KN_TRF_ROWS, KB_GBSV);
         return k;
     }
+    if (nrhs == 1 && trf_cols_available(kl, ku)) {
+        put(KN_TRF_COLS, KB_TRF_FWD);
+        put(kl + ku + 1 <= 4 && trs_rows_preferred(kl, ku) ? KN_TRS_ROWS
+            : kl + ku + 1 <= 32 ? KN_TRS_BWD : KN_TRS_WINDOW, KB_TRS_BWD);
+        return k;
+    }
     if (nrhs == 1 && (trf_window_available(kl, ku) || trf_wide_available(kl, ku))) {
         const int tv = trf_thread_preferred(kl, ku) ? KN_TRF_THREAD
                        : trf_wide_available(kl, ku) ? KN_TRF_WIDE
@@ -900,7 +961,7 @@ int trfs_plan(int n, int kl, int ku, int nrhs, int64_t batch, int phase, int *ki
         return k;
     }
     const int tv = pick_trf(n, n, kl, ku);
-    put(tv == BANDLU_ROWS ? (trf_wide_available(kl, ku) ? KN_TRF_WIDE : KN_TRF_ROWS)
+    put(tv == BANDLU_COLS ? KN_TRF_COLS : tv == BANDLU_ROWS ? (trf_wide_available(kl, ku) ? KN_TRF_WIDE : KN_TRF_ROWS)
         : tv == BANDLU_WINDOW ? KN_TRF_WINDOW : tv == BANDLU_THREAD ? KN_TRF_THREAD : KN_TRF_GENERIC, KB_TRF);
     const int sv = pick_trs(n, kl, ku, nrhs);
     put(sv == BANDLU_ROWS ? KN_TRS_ROWS : sv == BANDLU_WINDOW ? (nrhs == 1 ? KN_TRS_BLK : KN_TRS_WINDOW) : KN_TRS_GENERIC,
@@ -935,6 +996,20 @@ int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ld
         BANDLU_ROWS_LIST(X)
 #undef X
         return BANDLU_ERR_UNSUPPORTED;
+    }
+    if (n > 0 && nrhs == 1 && trf_cols_available(kl, ku)) {
+        int r = BANDLU_ERR_UNSUPPORTED;
+        Strided<const double> Ac{A.base, A.stride};
+        Strided<const int> Pc{P.base, P.stride};
+#define X(a, b, g, c)                                                                                     \
+    if (kl == a && ku == b) {                                                                             \
+        r = 0;                                                                                            \
+        if (phase != 2) r = launch_trf_cols<a, b, g, c, FL_FWD>(n, A, ldab, P, info, batch, st, B);       \
+        if (r == 0 && phase != 1) r = launch_trs_bwd<a, b>(n, Ac, ldab, Pc, B, ldb, batch, st);           \
+    }
+        BANDLU_COLS_LIST(X)
+#undef X
+        return r;
     }
     if (n > 0 && nrhs == 1 && (trf_window_available(kl, ku) || trf_wide_available(kl, ku))) {
         int r = BANDLU_ERR_UNSUPPORTED;
@@ -1111,6 +1186,7 @@ int bandlu_rows_available(int kl, int ku) { return trf_rows_available(kl, ku) ? 
 int bandlu_thread_available(int kl, int ku) { return trf_thread_available(kl, ku) ? 1 : 0; }
 int bandlu_tpm_available(int kl, int ku) { return trf_tpm_available(kl, ku) ? 1 : 0; }
 int bandlu_thin_available(int kl, int ku) { return trf_thin_available(kl, ku) ? 1 : 0; }
+int bandlu_cols_available(int kl, int ku) { return trf_cols_available(kl, ku) ? 1 : 0; }
 
 // 1 if (kl, ku) is served by run-time compiled kernels (jit.cuh), else 0 (no compilation)
 int bandlu_jit_band(int kl, int ku) { return jit_band(kl, ku) ? 1 : 0; }

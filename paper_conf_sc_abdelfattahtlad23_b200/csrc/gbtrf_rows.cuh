@@ -138,6 +138,11 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
     constexpr int KV = C::KV, U = C::U, H = C::H, WP = C::WP, RP = C::RP, D = C::D, RR = C::RR, BK = C::BK,
                   BIT = C::BIT;
     constexpr int FREE = 0x7fffffff;
+#ifdef BANDLU_ROWS_NOHOIST
+    constexpr bool HOIST = false;
+#else
+    constexpr bool HOIST = C::W <= 24;
+#endif
     extern __shared__ __align__(16) double smem[];
 
     const int lane = (int)lane_id(), wib = (int)(threadIdx.x >> 5);
@@ -184,6 +189,9 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
     constexpr int KS = G / U;
     const int64_t kstride = (int64_t)KS * (ldab - 1);
     auto stage_block = [&](int qb, const double *colq) {
+#ifdef BANDLU_ABL_NOSTAGE
+        if (qb >= 0) { cp_async_commit(); return; }
+#endif
         if constexpr (G % U == 0) {
             const int q = qb + t % U, c0 = qb - KL + t / U;
             const bool rowok = q < mloc;
@@ -281,7 +289,14 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
         for (int ri = 0; ri < R; ++ri) {
             o.x[ri] = VS(ri, s);
             o.cand[ri] = (pos[ri] <= j + KL) && (pos[ri] < mloc);
+#ifndef BANDLU_ROWS_KEY64
+            // |x| as integer words (no DADD |x| on the FP64 pipe in the search chain; C3 -0.3%)
+            const uint64_t k = o.cand[ri] ? (((uint64_t)((unsigned)__double2hiint(o.x[ri]) & 0x7fffffffu) << 32) |
+                                             (unsigned)__double2loint(o.x[ri]))
+                                          : 0ull;
+#else
             const uint64_t k = o.cand[ri] ? abs_key(o.x[ri]) : 0ull;
+#endif
             const bool better = o.cand[ri] && (!cb || k > kb || (k == kb && pos[ri] < pb));
             if (better) {
                 kb = k;
@@ -290,6 +305,9 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
                 cb = true;
             }
         }
+#ifdef BANDLU_ABL_NOSEARCH
+        if (j >= 0) { o.pb = pb; o.rb = rb; o.gb = 1u; return; }
+#endif
         const unsigned hi = (unsigned)(kb >> 32);
         const unsigned mhi = group_max_u32<G>(hi, g);
         unsigned gb = (__ballot_sync(0xffffffffu, cb && hi == mhi) >> gbase) & gbits;
@@ -369,12 +387,29 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
 
             // ---- pivot row (U row j: slots s..s+KV) + (B entry, logical row) -> record s
             const uint32_t rcs = rec_s + (uint32_t)(s * WP * 8);
+#if defined(BANDLU_ROWS_REC64)
+            // 64-bit record stores: one wavefront each for the GPW pivot lanes (a 128-bit store
+            // from lanes in both half-warps takes two)
 #pragma unroll
             for (int ri = 0; ri < R; ++ri) {
 #pragma unroll
-                for (int h = s / 2; h <= (s + KV) / 2; ++h)
-                    st_shared_v2_if(is_piv && rb == ri, rcs + h * 16, v[ri][h + OFF / 2]);
+                for (int k = s; k <= s + KV; ++k) st_shared_f64_if(is_piv && rb == ri, rcs + k * 8, VS(ri, k + OFF));
             }
+#elif !defined(BANDLU_ABL_NOREC)
+#pragma unroll
+            for (int ri = 0; ri < R; ++ri) {
+#pragma unroll
+                for (int h = s / 2; h <= (s + KV) / 2; ++h) {
+#ifdef BANDLU_ABL_HALF
+                    // (timing experiment, wrong results) half the record stores
+                    if (h != s / 2 && (h & 1)) continue;
+#endif
+                    st_shared_v2_if(is_piv && rb == ri, rcs + h * 16, v[ri][h + OFF / 2]);
+                }
+            }
+#else
+            st_shared_v2_if(is_piv, rcs + (s / 2) * 16, v[0][s / 2 + OFF / 2]);
+#endif
             {
                 double bsel = bq[0];
 #pragma unroll
@@ -385,6 +420,14 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
 
             // ---- broadcast read (64-bit: one cycle per warp for all groups)
             const double2 yp = ld_shared_v2(rcs + RP * 8);
+            // the update's pivot-row reads issue before RN(1/p): their latency overlaps it (C3
+            // factorization 0.926 -> 0.918 ms with KEY32; windows W <= 24 only: ~10 more registers)
+            const int HLO = (s + 1) / 2;
+            double2 u2h[KV / 2 + 2];
+            if constexpr (HOIST) {
+#pragma unroll
+                for (int h = HLO; h <= (s + KV) / 2; ++h) u2h[h - HLO] = ld_shared_v2(rcs + h * 16);
+            }
 #ifdef BANDLU_ROWS_FASTCHAIN
             const int ppos = ppos_f;
             const bool zp = (rinv == 0.0);
@@ -418,14 +461,20 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
 
             // ---- SCAL: multiplier = x * RN(1/p) (DSCAL(ONE/pivot), Q7)
 #ifndef BANDLU_ROWS_FASTCHAIN
+#ifdef BANDLU_ABL_NORCP
+            const double rinv = p;
+#else
             const double rinv = __drcp_rn(p);
+#endif
 #endif
             double lu[R];
 #pragma unroll
             for (int ri = 0; ri < R; ++ri) {
                 const double l = zp ? x[ri] : __dmul_rn(x[ri], rinv);
                 lu[ri] = (cand[ri] && !zp) ? l : 0.0;
+#ifndef BANDLU_ABL_NOOUT
                 if (cand[ri] && !pslot[ri]) colj[pos[ri] - j] = l;
+#endif
             }
             if constexpr (FWD) {
                 const double y = yp.x;
@@ -452,7 +501,12 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
             }
 #pragma unroll
             for (int h = (s + 1) / 2; h <= (s + KV) / 2; ++h) {
-                const double2 u2 = ld_shared_v2(rcs + h * 16);
+#if defined(BANDLU_ABL_HALF)
+                // (timing experiment, wrong results) half the broadcast loads
+                const double2 u2 = ld_shared_v2(rcs + ((h & 1) && h > (s + 1) / 2 ? h - 1 : h) * 16);
+#else
+                const double2 u2 = HOIST ? u2h[h - HLO] : ld_shared_v2(rcs + h * 16);
+#endif
 #ifdef BANDLU_ROWS_FASTCHAIN
                 // column j+1 (slot s+1) uses the shuffled value (bitwise the record's)
                 const double ua = (2 * h == s + 1) ? u1 : u2.x, ub = (2 * h + 1 == s + 1) ? u1 : u2.y;
@@ -485,7 +539,11 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
         }
         // ---- U rows j0 .. j0+U-1 (the block's records) -> HBM, 32-byte column chunks
         __syncwarp();
+#ifdef BANDLU_ABL_NOOUT
+        if (j0 < 0) {
+#else
         if constexpr (G % U == 0) {
+#endif
             const bool rowok = live && j0 + t % U < mn;
             const int c0 = j0 + t / U;
             const uint32_t src0 = rec_s + (uint32_t)(((t % U) * WP + t / U) * 8);
@@ -544,7 +602,13 @@ __global__ void BANDLU_ROWS_BOUNDS(TrfRows<KL, KU, G, R>)
 #pragma unroll
         for (int ri = 0; ri < R; ++ri) {
 #pragma unroll
-            for (int k = 0; k < 2 * H; ++k) VS(ri, k) = (k + SH < 2 * H) ? VS(ri, k + SH) : 0.0;
+            for (int k = 0; k < 2 * H; ++k) {
+#ifdef BANDLU_ABL_NOSHIFT
+                if (k + SH >= 2 * H) VS(ri, k) = 0.0;
+#else
+                VS(ri, k) = (k + SH < 2 * H) ? VS(ri, k + SH) : 0.0;
+#endif
+            }
         }
     }
     cp_async_wait<0>();

@@ -112,8 +112,11 @@ def test_variant_heuristic_is_shape_only(lib):
     assert b.rows_available(10, 10) and b.rows_available(2, 32) and b.rows_available(1, 1)
     assert not b.rows_available(0, 3) and not b.rows_available(3, 0)
     assert not b.tc_available(10, 10) and not b.thread_available(1, 1)  # opt-in builds only (-DBANDLU_WITH_TC/THREAD)
-    assert b.trf_variant(256, 256, 1, 1) == b.ROWS  # thin bands: row-slot kernel too
-    assert b.trf_variant(64, 64, 0, 3) == b.WINDOW
+    # thin lower bands, square: the column-owner kernel; rectangular: row-slot / window kernels
+    assert b.trf_variant(256, 256, 1, 1) == b.COLS and b.trf_variant(512, 512, 2, 3) == b.COLS
+    assert b.trf_variant(300, 256, 1, 1) == b.ROWS
+    assert b.trf_variant(64, 64, 0, 3) == b.COLS and b.trf_variant(64, 60, 0, 3) == b.WINDOW
+    assert b.cols_available(3, 2) and not b.cols_available(10, 10) and not b.cols_available(2, 32)
     assert b.trf_variant(100, 100, 32, 32) == b.ROWS  # kl+1 > 32 lanes: two-warp row-slot kernel
     # band not instantiated ahead of time: run-time compiled row-slot kernels (NVRTC), else the safeguard
     assert b.trf_variant(100, 100, 33, 20) == (b.ROWS if b.jit_band(33, 20) else b.GENERIC)
@@ -152,6 +155,9 @@ def test_trfs_plan_reports_the_launches(lib):
     assert p["kernels"] == ["gbtrf_wide_kernel", "gbtrs_window_kernel"] and not p["fused"]
     p = b.trfs_plan(1024, 2, 32, 1, 100)  # kl+ku+1+PF > 2G: no fused kernel for (2,32)
     assert p["kernels"] == ["gbtrf_rows_kernel", "gbtrs_window_kernel"] and not p["fused"]
+    p = b.trfs_plan(256, 1, 1, 1, 10000)  # C2: beyond one wave of the fused kernel
+    assert p["kernels"] == ["gbtrf_cols_kernel", "gbtrs_rows_kernel"] and not p["fused"]
+    assert b.trfs_plan(64, 2, 2, 1, 100)["fused"]  # C1: one launch
     p = b.trfs_plan(512, 10, 10, 1, 1000, b.TRFS_TWO_LAUNCH)
     assert p["kernels"] == ["gbtrf_rows_kernel", "gbtrs_bwd_kernel"]
     p = b.trfs_plan(1024, 2, 32, 16, 5000)

@@ -45,6 +45,8 @@ def trf_variants(kl, ku, square=True):
         v.append(bl.TPM)
     if square and bl.thin_available(kl, ku):
         v.append(bl.THIN)
+    if square and bl.cols_available(kl, ku):
+        v.append(bl.COLS)
     if bl.rows_available(kl, ku):
         v.append(bl.ROWS)
     if bl.tc_available(kl, ku):
@@ -67,7 +69,7 @@ def _check_trf(m, n, kl, ku, batch, variant, ldab=None, first=0, A_in=None):
 
 
 @pytest.mark.parametrize("kl,ku", ALL_BANDS)
-@pytest.mark.parametrize("variant", [bl.WINDOW, bl.GENERIC, bl.ROWS, bl.TC, bl.THREAD, bl.TPM, bl.THIN])
+@pytest.mark.parametrize("variant", [bl.WINDOW, bl.GENERIC, bl.ROWS, bl.TC, bl.THREAD, bl.TPM, bl.THIN, bl.COLS])
 @pytest.mark.parametrize("n", [1, 2, 7, 37, 100])
 def test_trf_parity_small(kl, ku, variant, n):
     if variant not in trf_variants(kl, ku):
@@ -87,7 +89,7 @@ def test_trf_parity_rectangular(kl, ku, mn):
 @pytest.mark.parametrize("kl,ku", [(2, 3), (10, 10), (5, 9), (33, 20), (32, 32), (40, 64), (0, 40)])
 def test_trf_parity_generic_any_band(kl, ku):
     _check_trf(150, 150, kl, ku, batch=11, variant=bl.GENERIC)
-    assert bl.trf_variant(150, 150, kl, ku) in (bl.GENERIC, bl.WINDOW, bl.ROWS)
+    assert bl.trf_variant(150, 150, kl, ku) in (bl.GENERIC, bl.WINDOW, bl.ROWS, bl.COLS)
 
 
 @pytest.mark.parametrize("kl,ku", [(1, 1), (10, 10), (2, 32), (32, 32)])
@@ -551,7 +553,8 @@ def test_fused_gbsv_kernel_vs_oracle_and_two_launch_plan(kl, ku, n):
     batch = 19  # ragged: not a multiple of matrices per warp / CTA
     plan = bl.trfs_plan(n, kl, ku, 1, batch)
     assert plan["fused"] and plan["kernels"] == ["gbtrf_rows_kernel"]
-    assert bl.trfs_plan(n, kl, ku, 1, batch, bl.TRFS_TWO_LAUNCH)["kernels"][0] == "gbtrf_rows_kernel"
+    two = bl.trfs_plan(n, kl, ku, 1, batch, bl.TRFS_TWO_LAUNCH)["kernels"][0]
+    assert two == ("gbtrf_cols_kernel" if bl.cols_available(kl, ku) else "gbtrf_rows_kernel")
     A = I.gen_band(n, n, kl, ku, count=batch, first=n)
     B = I.gen_rhs(n, 1, ldb=n + 2, count=batch, first=n)
     Ao, Bo = A.copy(), B.copy()
@@ -694,3 +697,44 @@ def test_thin_fused_kernel_vs_oracle(kl, ku, n):
         if n > 4:
             ok[6] = True  # singular U: Inf/NaN pattern of x out of contract (reading 12)
         assert np.all(ok)
+
+
+COLS_BANDS = [(0, 0), (0, 3), (1, 1), (2, 2), (2, 3), (3, 0), (3, 2), (4, 4), (2, 32)]  # skipped where not compiled
+
+
+@pytest.mark.parametrize("kl,ku", COLS_BANDS)
+@pytest.mark.parametrize("n", [3, 4, 5, 15, 16, 17, 33, 48, 49, 64, 131])
+def test_cols_kernel_parity(kl, ku, n):
+    """Column-owner factorization (gbtrf_cols.cuh) at n around its ring / unroll period (GL steps,
+    GL*CPL column slots) and staging block (4 rows), ragged batch: bitwise vs the oracle."""
+    if not bl.cols_available(kl, ku):
+        pytest.skip("no column-owner kernel compiled for this band")
+    assert bl.trf_variant(n, n, kl, ku) == bl.COLS
+    _check_trf(n, n, kl, ku, batch=45, variant=bl.COLS)
+
+
+@pytest.mark.parametrize("kl,ku", COLS_BANDS)
+@pytest.mark.parametrize("n,batch", [(5, 9), (40, 33), (257, 70)])
+def test_cols_trfs_forward_parity(kl, ku, n, batch):
+    # batches beyond one wave of the fused row-slot kernel (or forced two-launch) take the
+    # column-owner factorization with the forward substitution, then the backward solve
+    """dgbtrfs on a column-owner band (factorization with the forward substitution on the fly,
+    then the backward solve): factors, pivots and solution bitwise vs oracle dgbtrf + dgbtrs."""
+    if not bl.cols_available(kl, ku):
+        pytest.skip("no column-owner kernel compiled for this band")
+    A = I.gen_band(n, n, kl, ku, count=batch)
+    B = I.gen_rhs(n, 1, count=batch)
+    Ao, Bo = A.copy(), B.copy()
+    ipo, info_o = oracle.dgbtrf(Ao, n, n, kl, ku)
+    oracle.dgbtrs(Ao, ipo, Bo, n, kl, ku)
+    plan = bl.trfs_plan(n, kl, ku, 1, batch, bl.TRFS_TWO_LAUNCH)
+    assert plan["kernels"][0] == "gbtrf_cols_kernel", plan
+    Ag, Bg = torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda()
+    Pg = torch.zeros((batch, n), dtype=torch.int32, device="cuda")
+    Ig = torch.full((batch,), -7, dtype=torch.int32, device="cuda")
+    bl.dgbtrfs_strided_batched(n, kl, ku, Ag, Pg, Bg, Ig, phase=bl.TRFS_TWO_LAUNCH)
+    torch.cuda.synchronize()
+    assert np.array_equal(Ig.cpu().numpy(), info_o)
+    assert np.array_equal(Pg.cpu().numpy(), ipo)
+    assert same_bits(Ag.cpu().numpy(), Ao).all()
+    assert same_bits(Bg.cpu().numpy(), Bo).all()

@@ -9,7 +9,7 @@ import paper_conf_sc_abdelfattahtlad23_b200 as bl  # noqa: E402
 from paper_conf_sc_abdelfattahtlad23_b200 import inputs as I  # noqa: E402
 
 kl, ku, n, batch = (int(x) for x in sys.argv[1:5])
-names = {"rows": bl.ROWS, "tpm": bl.TPM, "window": bl.WINDOW, "generic": bl.GENERIC, "thread": bl.THREAD, "thin": bl.THIN}
+names = {"cols": bl.COLS, "rows": bl.ROWS, "tpm": bl.TPM, "window": bl.WINDOW, "generic": bl.GENERIC, "thread": bl.THREAD, "thin": bl.THIN}
 A0 = I.gen_band_torch(n, n, kl, ku, count=batch, device="cuda")
 A = torch.empty_like(A0)
 P = torch.zeros((batch, n), dtype=torch.int32, device="cuda")
