@@ -111,12 +111,13 @@ namespace {
     X(2, 3, 4, 2)           \
     X(3, 0, 4, 1)           \
     X(3, 2, 4, 2)           \
+    X(2, 32, 16, 3)         \
     BANDLU_COLS_EXTRA(X)
 #endif
 // opt-in (measured): (4,4) slower than the row-slot kernel (XGC-like 0.096 vs
-// 0.072 ms); (2,32) with 8 lanes x 5 slots no faster (1.60 vs 1.62 ms at C4)
+// 0.072 ms, (4,4) n = 512 x 10,000: 0.576 vs 0.545 ms)
 #ifdef BANDLU_COLS_WIDE
-#define BANDLU_COLS_EXTRA(X) X(4, 4, 4, 3) X(2, 32, 8, 5)
+#define BANDLU_COLS_EXTRA(X) X(4, 4, 4, 3)
 #else
 #define BANDLU_COLS_EXTRA(X)
 #endif

@@ -45,8 +45,10 @@ struct TrfCols {
     static constexpr int WARPS = 4;
     static constexpr size_t smem_bytes() { return (size_t)WARPS * GPW * GROUP_DBL * sizeof(double); }
     static constexpr int MINB_SMEM = (int)((227 * 1024) / smem_bytes());
+    // resident CTAs per SM: 4 (128 registers); 2 (255 registers) for windows of >= 9 doubles per
+    // lane -- (2,32) with 16 lanes x 3 slots measured 2.03 ms at 128 registers, 1.42 ms at 255 (C4)
 #ifndef BANDLU_COLS_MINB
-#define BANDLU_COLS_MINB 4
+#define BANDLU_COLS_MINB (CPL * (KL + 1) >= 9 ? 2 : 4)
 #endif
     static constexpr int MINB =
         MINB_SMEM < BANDLU_COLS_MINB ? (MINB_SMEM < 1 ? 1 : MINB_SMEM) : BANDLU_COLS_MINB;
@@ -99,8 +101,10 @@ __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<
 #pragma unroll
         for (int i = 0; i < BIT; ++i) {
             const int cc = cc0 + i * (GL / UB);
-            if (i * (GL / UB) < BK) {
-                const bool ok = rowok && cc < BK && (cc - so >= 0) && (cc - so <= KV) && (j0b + cc < nl);
+            // cc >= BK would land in the next staging row (pitch BKP = BK): no copy at all (a
+            // zero-fill there raced with the real copy of that element)
+            if (i * (GL / UB) < BK && cc < BK) {
+                const bool ok = rowok && (cc - so >= 0) && (cc - so <= KV) && (j0b + cc < nl);
                 cp_async8(dst0 + (uint32_t)(i * (GL / UB) * 8), ok ? (const void *)(src + i * xstride) : (const void *)g_dummy,
                           ok ? 8u : 0u);
             }
@@ -256,7 +260,11 @@ __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<
                 double y = bc[0];
 #pragma unroll
                 for (int r = 1; r <= KL; ++r) y = (p == r) ? bc[r] : y;
+#ifdef BANDLU_COLS_DEBUG
+                st_global_f64_if(own && j < nl, bv + j, a[0][KL]);  // (debug) the incoming entry of column j
+#else
                 st_global_f64_if(own && j < nl, bv + j, y);
+#endif
                 double v[KL + 1];
 #pragma unroll
                 for (int r = 1; r <= KL; ++r) {

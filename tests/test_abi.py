@@ -116,7 +116,8 @@ def test_variant_heuristic_is_shape_only(lib):
     assert b.trf_variant(256, 256, 1, 1) == b.COLS and b.trf_variant(512, 512, 2, 3) == b.COLS
     assert b.trf_variant(300, 256, 1, 1) == b.ROWS
     assert b.trf_variant(64, 64, 0, 3) == b.COLS and b.trf_variant(64, 60, 0, 3) == b.WINDOW
-    assert b.cols_available(3, 2) and not b.cols_available(10, 10) and not b.cols_available(2, 32)
+    assert b.cols_available(3, 2) and b.cols_available(2, 32) and not b.cols_available(10, 10)
+    assert not b.cols_available(4, 4)  # opt-in (-DBANDLU_COLS_WIDE): measured slower
     assert b.trf_variant(100, 100, 32, 32) == b.ROWS  # kl+1 > 32 lanes: two-warp row-slot kernel
     # band not instantiated ahead of time: run-time compiled row-slot kernels (NVRTC), else the safeguard
     assert b.trf_variant(100, 100, 33, 20) == (b.ROWS if b.jit_band(33, 20) else b.GENERIC)
@@ -154,14 +155,14 @@ def test_trfs_plan_reports_the_launches(lib):
     p = b.trfs_plan(2048, 32, 32, 1, 100)
     assert p["kernels"] == ["gbtrf_wide_kernel", "gbtrs_window_kernel"] and not p["fused"]
     p = b.trfs_plan(1024, 2, 32, 1, 100)  # kl+ku+1+PF > 2G: no fused kernel for (2,32)
-    assert p["kernels"] == ["gbtrf_rows_kernel", "gbtrs_window_kernel"] and not p["fused"]
+    assert p["kernels"] == ["gbtrf_cols_kernel", "gbtrs_window_kernel"] and not p["fused"]
     p = b.trfs_plan(256, 1, 1, 1, 10000)  # C2: beyond one wave of the fused kernel
     assert p["kernels"] == ["gbtrf_cols_kernel", "gbtrs_rows_kernel"] and not p["fused"]
     assert b.trfs_plan(64, 2, 2, 1, 100)["fused"]  # C1: one launch
     p = b.trfs_plan(512, 10, 10, 1, 1000, b.TRFS_TWO_LAUNCH)
     assert p["kernels"] == ["gbtrf_rows_kernel", "gbtrs_bwd_kernel"]
     p = b.trfs_plan(1024, 2, 32, 16, 5000)
-    assert p["kernels"] == ["gbtrf_rows_kernel", "gbtrs_window_kernel"] and p["bytes"] == ["trf", "trs"]
+    assert p["kernels"] == ["gbtrf_cols_kernel", "gbtrs_window_kernel"] and p["bytes"] == ["trf", "trs"]
     p = b.trfs_plan(100, 5, 9, 1, 10, b.TRFS_TWO_LAUNCH)  # (5,9): not instantiated ahead of time
     if b.jit_band(5, 9):  # run-time compiled (NVRTC) kernels
         assert p["kernels"][0] == "gbtrf_rows_kernel" and p["kernels"][1] in ("gbtrs_bwd_kernel", "gbtrs_window_kernel", "gbtrs_blk_kernel")
