@@ -267,14 +267,15 @@ int launch_trf_rows(int m, int n, AP A, int ldab, PP P, int *info, int batch, cu
 }
 
 template <int KL, int KU, int GL, int CPL, int FL, class AP, class PP, class BP>
-int launch_trf_cols(int n, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st, BP B) {
+int launch_trf_cols(int n, AP A, int ldab, PP P, int *info, int batch, cudaStream_t st, BP B, int nrhs = 0,
+                    int ldb = 1) {
     using C = TrfCols<KL, KU, GL, CPL>;
     auto k = gbtrf_cols_kernel<KL, KU, GL, CPL, FL, AP, PP, BP>;
     const size_t sm = C::smem_bytes();
     if (int r = set_smem(k, sm)) return r;
     const int64_t per_block = (int64_t)C::WARPS * C::GPW;
     const unsigned grid = (unsigned)((batch + per_block - 1) / per_block);
-    k<<<grid, C::WARPS * 32, sm, st>>>(n, A, ldab, P, info, batch, B);
+    k<<<grid, C::WARPS * 32, sm, st>>>(n, A, ldab, P, info, batch, B, nrhs, ldb);
     return cuda_ret(cudaGetLastError());
 }
 
@@ -374,6 +375,14 @@ bool trf_cols_available(int kl, int ku) {
     BANDLU_COLS_LIST(X)
 #undef X
     return false;
+}
+// right-hand sides the column-owner kernel can carry through its forward substitution (one per lane)
+int trf_cols_rhs(int kl, int ku) {
+#define X(a, b, g, c) \
+    if (kl == a && ku == b) return g;
+    BANDLU_COLS_LIST(X)
+#undef X
+    return 0;
 }
 
 bool trs_window_available(int kl, int ku) {
@@ -946,9 +955,10 @@ int trfs_plan(int n, int kl, int ku, int nrhs, int64_t batch, int phase, int *ki
         put(KN_TRF_ROWS, KB_GBSV);
         return k;
     }
-    if (nrhs == 1 && trf_cols_available(kl, ku)) {
+    if (nrhs <= trf_cols_rhs(kl, ku)) {
         put(KN_TRF_COLS, KB_TRF_FWD);
-        put(kl + ku + 1 <= 4 && trs_rows_preferred(kl, ku) ? KN_TRS_ROWS
+        put(nrhs > 1 ? KN_TRS_WINDOW
+            : kl + ku + 1 <= 4 && trs_rows_preferred(kl, ku) ? KN_TRS_ROWS
             : kl + ku + 1 <= 32 ? KN_TRS_BWD : KN_TRS_WINDOW, KB_TRS_BWD);
         return k;
     }
@@ -998,15 +1008,17 @@ int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ld
 #undef X
         return BANDLU_ERR_UNSUPPORTED;
     }
-    if (n > 0 && nrhs == 1 && trf_cols_available(kl, ku)) {
+    if (n > 0 && nrhs <= trf_cols_rhs(kl, ku)) {  // factorization + forward substitution, then backward
         int r = BANDLU_ERR_UNSUPPORTED;
         Strided<const double> Ac{A.base, A.stride};
         Strided<const int> Pc{P.base, P.stride};
-#define X(a, b, g, c)                                                                                     \
-    if (kl == a && ku == b) {                                                                             \
-        r = 0;                                                                                            \
-        if (phase != 2) r = launch_trf_cols<a, b, g, c, FL_FWD>(n, A, ldab, P, info, batch, st, B);       \
-        if (r == 0 && phase != 1) r = launch_trs_bwd<a, b>(n, Ac, ldab, Pc, B, ldb, batch, st);           \
+#define X(a, b, g, c)                                                                                       \
+    if (kl == a && ku == b) {                                                                               \
+        r = 0;                                                                                              \
+        if (phase != 2) r = launch_trf_cols<a, b, g, c, FL_FWD>(n, A, ldab, P, info, batch, st, B, nrhs, ldb); \
+        if (r == 0 && phase != 1)                                                                           \
+            r = nrhs == 1 ? launch_trs_bwd<a, b>(n, Ac, ldab, Pc, B, ldb, batch, st)                        \
+                          : launch_trs_window<a, b>(n, nrhs, Ac, ldab, Pc, B, ldb, nullptr, batch, st, 0);  \
     }
         BANDLU_COLS_LIST(X)
 #undef X

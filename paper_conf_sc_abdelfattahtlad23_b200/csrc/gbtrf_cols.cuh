@@ -4,8 +4,9 @@
 // What it computes: LAPACK DGBTF2 exactly (Sec. 5.1 pseudo-code
 // P:350-367, ju rule P:492-494, right-only swaps P:358/P:369-374), the same
 // fp64 operation sequence as the oracle => bitwise-equal factors, ipiv, info;
-// with FL_FWD also the forward substitution of one right-hand side (DGBTRS 'N'
-// first loop) on the fly, as gbtrf_rows.cuh does.
+// with FL_FWD also the forward substitution of nrhs <= GL right-hand sides (DGBTRS
+// 'N' first loop) on the fly: lane t carries right-hand side t as one
+// more column slot, so y never round-trips through HBM before the backward solve.
 //
 // Why ("gbtrf_cols"): the row-slot kernel gives every lane a
 // row of the window (kl+ku+1 doubles) and broadcasts the pivot row each step;
@@ -40,8 +41,9 @@ struct TrfCols {
     static constexpr int BKP = ((BK + 1) / 2) * 2;  // row pitch (doubles), 16-byte rows
     static constexpr int NSB = 4;                 // staging ring (pow2): two blocks ahead
     static constexpr int BIT = (BK * UB + GL - 1) / GL;
-    // per group: NSB staging blocks + one output block (UB x BKP each) + NSB x UB RHS entries
-    static constexpr int GROUP_DBL = (NSB + 1) * UB * BKP + NSB * UB;
+    // per group: NSB staging blocks + one output block (UB x BKP each) + NSB x UB x GL entries of
+    // the right-hand sides (FL_FWD: lane t carries right-hand side t, nrhs <= GL)
+    static constexpr int GROUP_DBL = (NSB + 1) * UB * BKP + NSB * UB * GL;
     static constexpr int WARPS = 4;
     static constexpr size_t smem_bytes() { return (size_t)WARPS * GPW * GROUP_DBL * sizeof(double); }
     static constexpr int MINB_SMEM = (int)((227 * 1024) / smem_bytes());
@@ -63,7 +65,7 @@ __device__ __forceinline__ uint64_t abs_key_w(double x) {
 
 template <int KL, int KU, int GL, int CPL, int FL, class AP, class PP, class BP>
 __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<KL, KU, GL, CPL>::MINB)
-    gbtrf_cols_kernel(int n, AP A, int ldab, PP P, int *__restrict__ info, int batch, BP Bv) {
+    gbtrf_cols_kernel(int n, AP A, int ldab, PP P, int *__restrict__ info, int batch, BP Bv, int nrhs, int ldb) {
     using C = TrfCols<KL, KU, GL, CPL>;
     constexpr bool FWD = FL & 1;
     constexpr int KV = C::KV, NR = C::NR, UB = C::UB, BK = C::BK, BKP = C::BKP, NSB = C::NSB, BIT = C::BIT;
@@ -78,7 +80,9 @@ __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<
     if (__ballot_sync(0xffffffffu, live) == 0u) return;
     double *__restrict__ ab = live ? A.get(mat) : g_dummy;
     int *__restrict__ ipiv = live ? P.get(mat) : nullptr;
-    double *__restrict__ bv = (FWD && live) ? Bv.get(mat) : g_dummy;
+    // FWD: lane t owns right-hand side t (t < nrhs <= GL), B(:, t) = bcol[0 .. n-1]
+    const bool rown = FWD && live && t < nrhs;
+    double *__restrict__ bcol = rown ? Bv.get(mat) + (int64_t)t * ldb : g_dummy;
     // loop control uses n (the same for every group of the warp); memory predicates use nl
     // (0 for dead groups, so they run the same instruction stream without touching memory)
     const int nl = live ? n : 0;
@@ -86,7 +90,7 @@ __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<
     double *grp = smem + (size_t)(wib * C::GPW + g) * C::GROUP_DBL;
     const uint32_t stage_s = smem_u32(grp);                              // NSB x [UB][BKP]
     const uint32_t out_s = stage_s + NSB * UB * BKP * 8;                 // [UB][BKP]
-    const uint32_t bst_s = out_s + UB * BKP * 8;                         // NSB x [UB] RHS entries
+    const uint32_t bst_s = out_s + UB * BKP * 8;                         // NSB x [UB][GL] RHS entries
 
     // ---- block transfers: lane t moves row offset so = t % UB, columns cc = t / UB + i * GL / UB
     const int so = t % UB, cc0 = t / UB;
@@ -109,12 +113,15 @@ __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<
                           ok ? 8u : 0u);
             }
         }
-        if constexpr (FWD) {
-            if (t < UB) {
-                const int q = j0b + KL + t;
-                const bool ok = q < nl;
-                cp_async8(bst_s + (uint32_t)(((b & (NSB - 1)) * UB + t) * 8),
-                          ok ? (const void *)(bv + q) : (const void *)g_dummy, ok ? 8u : 0u);
+        if constexpr (FWD) {  // rows q0 .. q0+3 of this lane's right-hand side (zeros past n / unowned)
+            // (16-byte pairs with the entries held in registers for the block measured slower: C4
+            // factorization + forward 1.99 vs 1.92 ms)
+#pragma unroll
+            for (int o = 0; o < UB; ++o) {
+                const int q = j0b + KL + o;
+                const bool ok = rown && q < nl;
+                cp_async8(bst_s + (uint32_t)((((b & (NSB - 1)) * UB + o) * GL + t) * 8),
+                          ok ? (const void *)(bcol + q) : (const void *)g_dummy, ok ? 8u : 0u);
             }
         }
         cp_async_commit();
@@ -140,7 +147,7 @@ __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<
 
     // ---- window registers: a[k][r] = A(j+r, c_k) for the column c_k of slot k
     double a[CPL][KL + 1];
-    double bc[KL + 1];  // FWD: the right-hand side entries of rows j..j+KL
+    double bc[KL + 1];  // FWD: entries j..j+KL of this lane's right-hand side
 #pragma unroll
     for (int k = 0; k < CPL; ++k) {
         const int c = k * GL + t;
@@ -151,7 +158,7 @@ __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<
         }
     }
 #pragma unroll
-    for (int r = 0; r <= KL; ++r) bc[r] = (FWD && r < KL && r < nl) ? bv[r] : 0.0;
+    for (int r = 0; r <= KL; ++r) bc[r] = (rown && r < KL && r < nl) ? bcol[r] : 0.0;
 
     stage_block(0);
     stage_block(1);
@@ -184,7 +191,7 @@ __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<
             }
             if constexpr (FWD) {
                 double x = 0.0;
-                ld_shared_f64_if(j + KL < nl, bst_s + (uint32_t)(((b & (NSB - 1)) * UB + o) * 8), x);
+                ld_shared_f64_if(rown, bst_s + (uint32_t)((((b & (NSB - 1)) * UB + o) * GL + t) * 8), x);
                 bc[KL] = x;
             }
 
@@ -256,15 +263,11 @@ __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<
                     for (int r = 0; r < KL; ++r) a[0][r] = 0.0;
                 }
             }
-            if constexpr (FWD) {  // the right-hand side column: same interchange, DGER zero skip
+            if constexpr (FWD) {  // the right-hand side columns: same interchange, DGER zero skip (per column)
                 double y = bc[0];
 #pragma unroll
                 for (int r = 1; r <= KL; ++r) y = (p == r) ? bc[r] : y;
-#ifdef BANDLU_COLS_DEBUG
-                st_global_f64_if(own && j < nl, bv + j, a[0][KL]);  // (debug) the incoming entry of column j
-#else
-                st_global_f64_if(own && j < nl, bv + j, y);
-#endif
+                st_global_f64_if(rown && j < nl, bcol + j, y);
                 double v[KL + 1];
 #pragma unroll
                 for (int r = 1; r <= KL; ++r) {

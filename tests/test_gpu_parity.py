@@ -715,20 +715,23 @@ def test_cols_kernel_parity(kl, ku, n):
 
 @pytest.mark.parametrize("kl,ku", COLS_BANDS)
 @pytest.mark.parametrize("n,batch", [(5, 9), (40, 33), (257, 70)])
-def test_cols_trfs_forward_parity(kl, ku, n, batch):
+@pytest.mark.parametrize("nrhs", [1, 3, 4, 16])
+def test_cols_trfs_forward_parity(kl, ku, n, batch, nrhs):
     # batches beyond one wave of the fused row-slot kernel (or forced two-launch) take the
     # column-owner factorization with the forward substitution, then the backward solve
     """dgbtrfs on a column-owner band (factorization with the forward substitution on the fly,
     then the backward solve): factors, pivots and solution bitwise vs oracle dgbtrf + dgbtrs."""
     if not bl.cols_available(kl, ku):
         pytest.skip("no column-owner kernel compiled for this band")
+    if nrhs > 4 and (kl, ku) != (2, 32):
+        pytest.skip("4 lanes per matrix: up to 4 right-hand sides ride with the factorization")
     A = I.gen_band(n, n, kl, ku, count=batch)
-    B = I.gen_rhs(n, 1, count=batch)
+    B = I.gen_rhs(n, nrhs, ldb=n + 3, count=batch)  # NaN padding rows below each column stay untouched
     Ao, Bo = A.copy(), B.copy()
     ipo, info_o = oracle.dgbtrf(Ao, n, n, kl, ku)
     oracle.dgbtrs(Ao, ipo, Bo, n, kl, ku)
-    plan = bl.trfs_plan(n, kl, ku, 1, batch, bl.TRFS_TWO_LAUNCH)
-    assert plan["kernels"][0] == "gbtrf_cols_kernel", plan
+    plan = bl.trfs_plan(n, kl, ku, nrhs, batch, bl.TRFS_TWO_LAUNCH)
+    assert plan["kernels"][0] == "gbtrf_cols_kernel" and plan["bytes"] == ["trf_fwd", "trs_bwd"], plan
     Ag, Bg = torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda()
     Pg = torch.zeros((batch, n), dtype=torch.int32, device="cuda")
     Ig = torch.full((batch,), -7, dtype=torch.int32, device="cuda")
