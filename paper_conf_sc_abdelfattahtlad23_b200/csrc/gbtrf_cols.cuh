@@ -168,32 +168,42 @@ __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<
     for (int o = 0; o < UB; ++o) pv[o] = 0;
     double *lcol = ab + KV;  // &AB(KV, j): the multipliers of column j follow
 
+    // ---- the entries of row j+KL (position KL at step j), read from the staging block one step
+    // ahead so that the shared-memory latency is off the step's chain.  sn = the step's offset in
+    // its ring turn (j0 = j - sn); the column of slot k at that step:
+    double inc[CPL], incb = 0.0;
+    auto fetch_incoming = [&](int j, int sn, int j0) {
+        const int o = j % UB, b = j / UB;
+        const uint32_t srow = stage_s + (uint32_t)((((b & (NSB - 1)) * UB + o) * BKP - (j - o)) * 8);
+#pragma unroll
+        for (int k = 0; k < CPL; ++k) {
+            const int c = (k == 0 && t < sn) ? j0 + NR + t : j0 + k * GL + t;  // slot 0 of lanes < sn: next turn
+            const bool ok = (c - j <= KV) && (j + KL < nl) && (c < nl);
+            double x = 0.0;
+            ld_shared_f64_if(ok, srow + (uint32_t)(c * 8), x);
+            inc[k] = x;
+        }
+        if constexpr (FWD) {
+            double x = 0.0;
+            ld_shared_f64_if(rown, bst_s + (uint32_t)((((b & (NSB - 1)) * UB + o) * GL + t) * 8), x);
+            incb = x;
+        }
+    };
+    cp_async_wait<1>();  // block 0 landed
+    __syncwarp();
+    fetch_incoming(0, 0, 0);
+
 #pragma unroll 1
     for (int j0 = 0; j0 < n; j0 += GL) {
 #pragma unroll
         for (int s = 0; s < GL; ++s) {
             const int j = j0 + s, o = s % UB, b = j / UB;
             if (j >= n) break;
-            if (o == 0) {
-                stage_block(b + 2);
-                cp_async_wait<2>();
-                __syncwarp();
-            }
-            const uint32_t srow = stage_s + (uint32_t)((((b & (NSB - 1)) * UB + o) * BKP - (j - o)) * 8);
+            if (o == 0) stage_block(b + 2);
             // ---- row j+KL enters as position KL (zero outside its band / beyond n)
 #pragma unroll
-            for (int k = 0; k < CPL; ++k) {
-                const int c = (k == 0 && t < s) ? j0 + NR + t : j0 + k * GL + t;  // slot 0 of lanes < s: next ring turn
-                const bool ok = (c - j <= KV) && (j + KL < nl) && (c < nl);
-                double x = 0.0;
-                ld_shared_f64_if(ok, srow + (uint32_t)(c * 8), x);
-                a[k][KL] = x;
-            }
-            if constexpr (FWD) {
-                double x = 0.0;
-                ld_shared_f64_if(rown, bst_s + (uint32_t)((((b & (NSB - 1)) * UB + o) * GL + t) * 8), x);
-                bc[KL] = x;
-            }
+            for (int k = 0; k < CPL; ++k) a[k][KL] = inc[k];
+            if constexpr (FWD) bc[KL] = incb;
 
             // ---- owner of column j (lane s, slot 0): IAMAX (first max |x|, exact keys), RN(1/pivot)
 #ifdef BANDLU_COLS_SPEC
@@ -272,7 +282,7 @@ __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<
 #pragma unroll
                 for (int r = 1; r <= KL; ++r) {
                     v[r] = (p == r) ? bc[0] : bc[r];
-                    if (y != 0.0) v[r] = __fma_rn(e[r], -y, v[r]);
+                    fma_rn_if(y != 0.0, e[r], -y, v[r]);
                 }
 #pragma unroll
                 for (int r = 1; r <= KL; ++r) bc[r - 1] = v[r];
@@ -290,6 +300,15 @@ __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<
                             if (q <= o) ip[q] = pv[q];
                     }
                 }
+            }
+            // ---- next step's incoming entries (its block landed: wait for it at this block's end)
+            if (j + 1 < n) {
+                if (o == UB - 1) {
+                    cp_async_wait<1>();
+                    __syncwarp();
+                }
+                if (s + 1 < GL) fetch_incoming(j + 1, s + 1, j0);
+                else fetch_incoming(j + 1, 0, j0 + GL);  // the next ring turn (slots rotate below)
             }
         }
         // ---- ring turn: slot k <- slot k+1, the retired slot 0 (columns j0+NR+t) goes last
