@@ -12,10 +12,10 @@ import subprocess
 import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-OUT = os.path.join(ROOT, "gpurun_out")
+OUT = os.environ.get("NCU_DIR") or os.path.join(ROOT, "gpurun_out")  # where full_<cfg>.ncu-rep live
 PROF = os.environ.get("PROF_DIR") or os.path.join(ROOT, "profiles")  # the GPU box writes into gpurun_out/
 
-KERNELS = ("gbtrf_tpm_kernel", "gbtrf_rows_kernel", "gbtrf_window_kernel", "gbtrf_wide_kernel", "gbtrf_tc_kernel", "gbtrf_generic_kernel",
+KERNELS = ("gbtrf_tpm_kernel", "gbtrf_cols_kernel", "gbtrf_rows_kernel", "gbtrf_window_kernel", "gbtrf_wide_kernel", "gbtrf_tc_kernel", "gbtrf_generic_kernel",
            "gbtrs_window_kernel", "gbtrs_bwd_kernel", "gbtrs_rows_kernel", "gbtrs_generic_kernel", "gbtrs_t_generic_kernel",
            "gbtrs_blk_kernel", "gbtrs_t_kernel")
 KEYS = {
