@@ -42,15 +42,26 @@ struct FusedSolve {
     // two rows per lane suffice and the staging ring has PF steps before a row is used
     static constexpr bool ok = (KV + 1 + PF <= 2 * G) && (G % PF == 0 || PF % G == 0) && G >= 2;
 };
+// [r2b] the largest prefetch distance PF <= BANDLU_FUSED_PF (a power of two) that still satisfies
+// the constraints: small groups (the column-owner kernel's 4 lanes) with a shorter lead
+template <int KV, int G>
+struct FusedSolveAny {
+    static constexpr int pf(int x) {
+        return x < 1 ? 0 : ((KV + 1 + x <= 2 * G) && (G % x == 0 || x % G == 0)) ? x : pf(x / 2);
+    }
+    static constexpr int PF = pf(BANDLU_FUSED_PF);
+    static constexpr bool ok = PF > 0 && G >= 2;
+};
 
 // YSM: y(i) read from shared memory at ybuf_s + 8 i (else from bx[i], where the
 // forward pass left it).  wr: this group stores x into bx (false for dead
 // groups and, for dgbsv, where info > 0).  All 32 lanes of the warp call.
-template <int KV, int G, bool YSM>
+template <int KV, int G, bool YSM, int PF_ = FusedSolve<KV, G>::PF>
 __device__ __forceinline__ void backsolve_group(int n, const double *ab, int ldab, double *bx, uint32_t ybuf_s,
                                                 bool live, bool wr, int t, int gbase) {
-    constexpr int PF = FusedSolve<KV, G>::PF;
-    static_assert(FusedSolve<KV, G>::ok, "fused backward solve: needs kv + 1 + PF <= 2G");
+    constexpr int PF = PF_;
+    static_assert((KV + 1 + PF <= 2 * G) && (G % PF == 0 || PF % G == 0) && G >= 2,
+                  "fused backward solve: needs kv + 1 + PF <= 2G");
     constexpr unsigned FULL = 0xffffffffu;
     constexpr int NR = PF > G ? PF : G;  // ring period (unroll)
     auto yload = [&](bool p, int r, double &v) {  // predicated: v unchanged where !p

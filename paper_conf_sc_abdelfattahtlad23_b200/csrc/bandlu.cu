@@ -376,6 +376,20 @@ bool trf_cols_available(int kl, int ku) {
 #undef X
     return false;
 }
+// the column-owner kernel with the fused backward solve (nrhs = 1): one launch for dgbtrfs.
+// Opt-in (-DBANDLU_COLS_FUSED): bitwise, but the 4-lane backward pass (y re-read from B, prefetch
+// distance 2-4 steps) measured slower than the separate backward kernel: C2 0.59 vs 0.245 ms,
+// C1 0.049 vs 0.034 ms (the row-slot fused kernel).
+bool trf_cols_fused(int kl, int ku) {
+#ifdef BANDLU_COLS_FUSED
+#define X(a, b, g, c) \
+    if (kl == a && ku == b) return FusedSolveAny<a + b, g>::ok;
+    BANDLU_COLS_LIST(X)
+#undef X
+#endif
+    (void)kl, (void)ku;
+    return false;
+}
 // right-hand sides the column-owner kernel can carry through its forward substitution (one per lane)
 int trf_cols_rhs(int kl, int ku) {
 #define X(a, b, g, c) \
@@ -898,10 +912,18 @@ int64_t rows_wave(int kl, int ku) {
 #undef X
     return 0;
 }
+// dgbtrfs, nrhs = 1, a column-owner band: the column-owner kernel with the forward and backward
+// substitutions in the same launch (AUTO; TRFS_FUSED forces the row-slot fused kernel instead,
+// TRFS_TWO_LAUNCH the column-owner factorization + a backward launch)
+bool cols_fused_pick(int n, int kl, int ku, int nrhs, int phase) {
+    return n > 0 && nrhs == 1 && trf_cols_fused(kl, ku) && !(phase & (TRFS_TWO_LAUNCH | TRFS_FUSED));
+}
+
 bool trfs_fused_pick(int n, int kl, int ku, int nrhs, int64_t batch, int phase) {
     if (n <= 0 || nrhs != 1 || !rows_fused_available(kl, ku)) return false;
     if (phase & TRFS_TWO_LAUNCH) return false;
     if (phase & TRFS_FUSED) return true;
+    if (cols_fused_pick(n, kl, ku, nrhs, phase)) return false;
     return batch <= rows_wave(kl, ku);
 }
 
@@ -951,11 +973,15 @@ int trfs_plan(int n, int kl, int ku, int nrhs, int64_t batch, int phase, int *ki
             return k;
         }
     }
+    if (cols_fused_pick(n, kl, ku, nrhs, phase)) {
+        put(KN_TRF_COLS, KB_GBSV);
+        return k;
+    }
     if (trfs_fused_pick(n, kl, ku, nrhs, batch, phase)) {
         put(KN_TRF_ROWS, KB_GBSV);
         return k;
     }
-    if (nrhs <= trf_cols_rhs(kl, ku)) {
+    if (nrhs > 1 && nrhs <= trf_cols_rhs(kl, ku)) {
         put(KN_TRF_COLS, KB_TRF_FWD);
         put(nrhs > 1 ? KN_TRS_WINDOW
             : kl + ku + 1 <= 4 && trs_rows_preferred(kl, ku) ? KN_TRS_ROWS
@@ -993,8 +1019,20 @@ int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ld
     }
     phase &= ~TRFS_THIN;
     const bool fused = trfs_fused_pick(n, kl, ku, nrhs, batch, phase);
+    const bool cfused = cols_fused_pick(n, kl, ku, nrhs, phase);
     const int pflags = phase & (TRFS_TWO_LAUNCH | TRFS_FUSED);
     phase &= ~(TRFS_TWO_LAUNCH | TRFS_FUSED);
+    if (cfused) {
+        if (phase == 2) return 0;  // one launch
+#define X(a, b, g, c)                                                                                             \
+    if (kl == a && ku == b) {                                                                                     \
+        if constexpr (FusedSolveAny<a + b, g>::ok)                                                                \
+            return launch_trf_cols<a, b, g, c, FL_FWD | FL_BWD>(n, A, ldab, P, info, batch, st, B, nrhs, ldb);   \
+    }
+        BANDLU_COLS_LIST(X)
+#undef X
+        return BANDLU_ERR_UNSUPPORTED;
+    }
     if (fused) {
         if (phase == 2) return 0;  // the whole path is the first (only) launch
         const bool ysm = rows_ysm_fits_rt(n, kl, ku);
@@ -1008,7 +1046,11 @@ int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ld
 #undef X
         return BANDLU_ERR_UNSUPPORTED;
     }
-    if (n > 0 && nrhs <= trf_cols_rhs(kl, ku)) {  // factorization + forward substitution, then backward
+    // several right-hand sides on a column-owner band: factorization + forward substitution of all of
+    // them, then the backward solve (C4: 3.48 -> 3.19 ms).  One right-hand side keeps the row-slot /
+    // window kernels' forward-fused factorization: the column-owner one measured no faster there
+    // (C2 0.148 vs 0.145 ms, C5's (2,3) points 211 vs 204 ms), unlike plain dgbtrf (0.100 vs 0.133)
+    if (n > 0 && nrhs > 1 && nrhs <= trf_cols_rhs(kl, ku)) {
         int r = BANDLU_ERR_UNSUPPORTED;
         Strided<const double> Ac{A.base, A.stride};
         Strided<const int> Pc{P.base, P.stride};

@@ -26,6 +26,7 @@
 // blocks ahead); U rows leave the same way, one 4-row block at a time; the
 // multipliers are stored by the owner lane.
 #pragma once
+#include "backsolve_fused.cuh"
 #include "common.cuh"
 
 namespace bandlu {
@@ -67,7 +68,8 @@ template <int KL, int KU, int GL, int CPL, int FL, class AP, class PP, class BP>
 __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<KL, KU, GL, CPL>::MINB)
     gbtrf_cols_kernel(int n, AP A, int ldab, PP P, int *__restrict__ info, int batch, BP Bv, int nrhs, int ldb) {
     using C = TrfCols<KL, KU, GL, CPL>;
-    constexpr bool FWD = FL & 1;
+    constexpr bool FWD = FL & 1, BWD = FL & 2;  // FL_FWD, FL_BWD (gbtrf_rows.cuh)
+    static_assert(!BWD || (FWD && FusedSolveAny<KL + KU, GL>::ok), "fused backward solve");
     constexpr int KV = C::KV, NR = C::NR, UB = C::UB, BK = C::BK, BKP = C::BKP, NSB = C::NSB, BIT = C::BIT;
     static_assert((NSB & (NSB - 1)) == 0, "staging ring");
     extern __shared__ __align__(16) double smem[];
@@ -321,6 +323,12 @@ __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<
         }
     }
     cp_async_wait<0>();
+    if constexpr (BWD) {  // [r2b] the fused gbsv kernel: U x = y by the same lanes (one right-hand side,
+        // y(j) left in B(:,0) by lane 0, the U rows flushed above; backsolve_fused.cuh)
+        __syncwarp();
+        backsolve_group<KV, GL, false, FusedSolveAny<KV, GL>::PF>(n, ab, ldab, live ? Bv.get(mat) : g_dummy, 0u,
+                                                                  live, live, t, gbase);
+    }
     if (live && t == 0) info[mat] = (n > 0) ? linfo : 0;
 }
 

@@ -552,9 +552,10 @@ def _trfs(A_np, B_np, n, kl, ku, phase=0):
 def test_fused_gbsv_kernel_vs_oracle_and_two_launch_plan(kl, ku, n):
     batch = 19  # ragged: not a multiple of matrices per warp / CTA
     plan = bl.trfs_plan(n, kl, ku, 1, batch)
-    assert plan["fused"] and plan["kernels"] == ["gbtrf_rows_kernel"]
+    assert plan["fused"] and plan["kernels"][0] in ("gbtrf_rows_kernel", "gbtrf_cols_kernel")
+    assert bl.trfs_plan(n, kl, ku, 1, batch, bl.TRFS_FUSED)["kernels"] == ["gbtrf_rows_kernel"]
     two = bl.trfs_plan(n, kl, ku, 1, batch, bl.TRFS_TWO_LAUNCH)["kernels"][0]
-    assert two == ("gbtrf_cols_kernel" if bl.cols_available(kl, ku) else "gbtrf_rows_kernel")
+    assert two == "gbtrf_rows_kernel"  # one right-hand side: the row-slot forward-fused factorization
     A = I.gen_band(n, n, kl, ku, count=batch, first=n)
     B = I.gen_rhs(n, 1, ldb=n + 2, count=batch, first=n)
     Ao, Bo = A.copy(), B.copy()
@@ -717,8 +718,8 @@ def test_cols_kernel_parity(kl, ku, n):
 @pytest.mark.parametrize("n,batch", [(5, 9), (40, 33), (257, 70)])
 @pytest.mark.parametrize("nrhs", [1, 3, 4, 16])
 def test_cols_trfs_forward_parity(kl, ku, n, batch, nrhs):
-    # batches beyond one wave of the fused row-slot kernel (or forced two-launch) take the
-    # column-owner factorization with the forward substitution, then the backward solve
+    # nrhs > 1: the column-owner factorization with the forward substitution of all right-hand
+    # sides, then the backward solve; nrhs = 1: the row-slot / window plan (parity either way)
     """dgbtrfs on a column-owner band (factorization with the forward substitution on the fly,
     then the backward solve): factors, pivots and solution bitwise vs oracle dgbtrf + dgbtrs."""
     if not bl.cols_available(kl, ku):
@@ -731,7 +732,9 @@ def test_cols_trfs_forward_parity(kl, ku, n, batch, nrhs):
     ipo, info_o = oracle.dgbtrf(Ao, n, n, kl, ku)
     oracle.dgbtrs(Ao, ipo, Bo, n, kl, ku)
     plan = bl.trfs_plan(n, kl, ku, nrhs, batch, bl.TRFS_TWO_LAUNCH)
-    assert plan["kernels"][0] == "gbtrf_cols_kernel" and plan["bytes"] == ["trf_fwd", "trs_bwd"], plan
+    assert plan["bytes"] == ["trf_fwd", "trs_bwd"], plan
+    if nrhs > 1:  # the right-hand sides ride with the column-owner factorization
+        assert plan["kernels"][0] == "gbtrf_cols_kernel", plan
     Ag, Bg = torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda()
     Pg = torch.zeros((batch, n), dtype=torch.int32, device="cuda")
     Ig = torch.full((batch,), -7, dtype=torch.int32, device="cuda")
@@ -741,3 +744,21 @@ def test_cols_trfs_forward_parity(kl, ku, n, batch, nrhs):
     assert np.array_equal(Pg.cpu().numpy(), ipo)
     assert same_bits(Ag.cpu().numpy(), Ao).all()
     assert same_bits(Bg.cpu().numpy(), Bo).all()
+
+
+@pytest.mark.parametrize("kl,ku", [(0, 0), (0, 3), (1, 1), (2, 2), (2, 3), (3, 0), (3, 2)])
+@pytest.mark.parametrize("n,batch", [(1, 5), (3, 9), (8, 17), (63, 33), (256, 300)])
+def test_cols_fused_gbsv_kernel(kl, ku, n, batch):
+    """dgbtrfs in ONE launch on a column-owner band (factorization, forward and backward
+    substitution by the same lanes): factors, pivots, info and x bitwise vs the oracle, the NaN
+    ldb padding untouched; n from 1 (no step) to 256, batches not a multiple of 8 per warp."""
+    if not bl.cols_available(kl, ku) or bl.trfs_plan(n, kl, ku, 1, batch)["kernels"] != ["gbtrf_cols_kernel"]:
+        pytest.skip("column-owner fused kernel not built (opt-in -DBANDLU_COLS_FUSED)")
+    A = I.gen_band(n, n, kl, ku, count=batch, first=7)
+    B = I.gen_rhs(n, 1, ldb=n + 2, count=batch, first=7)
+    Ao, Bo = A.copy(), B.copy()
+    ipo, info_o = oracle.dgbtrf(Ao, n, n, kl, ku)
+    oracle.dgbtrs(Ao, ipo, Bo, n, kl, ku)
+    Ag, Pg, Bg, Ig = _trfs(A.copy(), B.copy(), n, kl, ku, 0)
+    assert np.array_equal(Ig, info_o) and np.array_equal(Pg, ipo)
+    assert np.all(same_bits(Ag, Ao)) and np.all(same_bits(Bg, Bo))
