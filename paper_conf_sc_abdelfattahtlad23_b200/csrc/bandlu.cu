@@ -390,6 +390,9 @@ bool trf_cols_fused(int kl, int ku) {
     (void)kl, (void)ku;
     return false;
 }
+#ifndef BANDLU_COLS_MIN_NRHS
+#define BANDLU_COLS_MIN_NRHS 1  // 2: one right-hand side keeps the row-slot / window plan
+#endif
 // right-hand sides the column-owner kernel can carry through its forward substitution (one per lane)
 int trf_cols_rhs(int kl, int ku) {
 #define X(a, b, g, c) \
@@ -981,7 +984,7 @@ int trfs_plan(int n, int kl, int ku, int nrhs, int64_t batch, int phase, int *ki
         put(KN_TRF_ROWS, KB_GBSV);
         return k;
     }
-    if (nrhs > 1 && nrhs <= trf_cols_rhs(kl, ku)) {
+    if (nrhs >= BANDLU_COLS_MIN_NRHS && nrhs <= trf_cols_rhs(kl, ku)) {
         put(KN_TRF_COLS, KB_TRF_FWD);
         put(nrhs > 1 ? KN_TRS_WINDOW
             : kl + ku + 1 <= 4 && trs_rows_preferred(kl, ku) ? KN_TRS_ROWS
@@ -1046,11 +1049,10 @@ int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ld
 #undef X
         return BANDLU_ERR_UNSUPPORTED;
     }
-    // several right-hand sides on a column-owner band: factorization + forward substitution of all of
-    // them, then the backward solve (C4: 3.48 -> 3.19 ms).  One right-hand side keeps the row-slot /
-    // window kernels' forward-fused factorization: the column-owner one measured no faster there
-    // (C2 0.148 vs 0.145 ms, C5's (2,3) points 211 vs 204 ms), unlike plain dgbtrf (0.100 vs 0.133)
-    if (n > 0 && nrhs > 1 && nrhs <= trf_cols_rhs(kl, ku)) {
+    // a column-owner band beyond one wave of the fused row-slot kernel: factorization + forward
+    // substitution of up to GL right-hand sides, then the backward solve (C4: 3.48 -> 3.19 ms; C2's
+    // factorization + forward 0.144 -> 0.135 ms once y is stored per 4-row block)
+    if (n > 0 && nrhs >= BANDLU_COLS_MIN_NRHS && nrhs <= trf_cols_rhs(kl, ku)) {
         int r = BANDLU_ERR_UNSUPPORTED;
         Strided<const double> Ac{A.base, A.stride};
         Strided<const int> Pc{P.base, P.stride};

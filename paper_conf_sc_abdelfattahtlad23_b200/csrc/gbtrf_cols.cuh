@@ -150,6 +150,10 @@ __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<
     // ---- window registers: a[k][r] = A(j+r, c_k) for the column c_k of slot k
     double a[CPL][KL + 1];
     double bc[KL + 1];  // FWD: entries j..j+KL of this lane's right-hand side
+    double yv[UB];      // FWD: y(j0b .. j0b+3) of this lane's right-hand side, stored per block
+#pragma unroll
+    for (int o = 0; o < UB; ++o) yv[o] = 0.0;
+    const bool a16y = ((reinterpret_cast<uintptr_t>(bcol) & 15) == 0);
 #pragma unroll
     for (int k = 0; k < CPL; ++k) {
         const int c = k * GL + t;
@@ -205,7 +209,9 @@ __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<
             // ---- row j+KL enters as position KL (zero outside its band / beyond n)
 #pragma unroll
             for (int k = 0; k < CPL; ++k) a[k][KL] = inc[k];
+#ifndef BANDLU_ABL_NOBIN
             if constexpr (FWD) bc[KL] = incb;
+#endif
 
             // ---- owner of column j (lane s, slot 0): IAMAX (first max |x|, exact keys), RN(1/pivot)
 #ifdef BANDLU_COLS_SPEC
@@ -279,7 +285,11 @@ __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<
                 double y = bc[0];
 #pragma unroll
                 for (int r = 1; r <= KL; ++r) y = (p == r) ? bc[r] : y;
+#ifdef BANDLU_COLS_YSTEP
                 st_global_f64_if(rown && j < nl, bcol + j, y);
+#else
+                yv[o] = y;  // stored per 4-row block (a store per step cost 17% at C2)
+#endif
                 double v[KL + 1];
 #pragma unroll
                 for (int r = 1; r <= KL; ++r) {
@@ -292,6 +302,20 @@ __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<
             // ---- block end: U rows and pivots of the 4 steps
             if (o == UB - 1 || j + 1 == n) {
                 flush_block(b);
+#ifndef BANDLU_COLS_YSTEP
+                if constexpr (FWD) {
+                    double *yd = bcol + (j - o);
+                    if (o == UB - 1 && a16y) {  // predicated-off lanes move nothing
+                        if (rown) {
+                            reinterpret_cast<double2 *>(yd)[0] = make_double2(yv[0], yv[1 % UB]);
+                            reinterpret_cast<double2 *>(yd)[1] = make_double2(yv[2 % UB], yv[3 % UB]);
+                        }
+                    } else {
+#pragma unroll
+                        for (int q = 0; q < UB; ++q) st_global_f64_if(rown && q <= o, yd + q, yv[q]);
+                    }
+                }
+#endif
                 if (live && t == 0) {
                     int *ip = ipiv + (j - o);
                     if (o == UB - 1 && (reinterpret_cast<uintptr_t>(ip) & 15) == 0) {

@@ -155,11 +155,11 @@ def test_trfs_plan_reports_the_launches(lib):
     p = b.trfs_plan(2048, 32, 32, 1, 100)
     assert p["kernels"] == ["gbtrf_wide_kernel", "gbtrs_window_kernel"] and not p["fused"]
     p = b.trfs_plan(1024, 2, 32, 1, 100)  # kl+ku+1+PF > 2G: no fused kernel for (2,32)
-    assert p["kernels"] == ["gbtrf_rows_kernel", "gbtrs_window_kernel"] and not p["fused"]
-    # C2 (beyond one wave of the row-slot fused kernel): two launches; C1: one.  One right-hand side
-    # keeps the row-slot forward-fused factorization (the column-owner one: plain dgbtrf, nrhs > 1)
+    assert p["kernels"] == ["gbtrf_cols_kernel", "gbtrs_window_kernel"] and not p["fused"]
+    # C2 (beyond one wave of the row-slot fused kernel): column-owner factorization + forward, then
+    # the backward kernel; C1 (within one wave): the row-slot fused kernel, one launch
     p = b.trfs_plan(256, 1, 1, 1, 10000)
-    assert p["kernels"] == ["gbtrf_rows_kernel", "gbtrs_rows_kernel"] and not p["fused"]
+    assert p["kernels"] == ["gbtrf_cols_kernel", "gbtrs_rows_kernel"] and not p["fused"]
     assert b.trfs_plan(256, 1, 1, 4, 10000)["kernels"] == ["gbtrf_cols_kernel", "gbtrs_window_kernel"]
     assert b.trfs_plan(64, 2, 2, 1, 100)["kernels"] == ["gbtrf_rows_kernel"]
     assert b.trfs_plan(256, 1, 1, 1, 10000, b.TRFS_FUSED)["kernels"] == ["gbtrf_rows_kernel"]

@@ -184,8 +184,9 @@ def test_gbsv_parity_with_singular(kl, ku, nrhs):
     assert np.array_equal(Bgn[3], B[3])  # untouched where info > 0
 
 
-def test_pointer_array_variants_match_strided():
-    n, kl, ku, nrhs, batch = 50, 10, 10, 2, 9
+@pytest.mark.parametrize("kl,ku", [(10, 10), (1, 1), (2, 32)])  # row-slot and column-owner (AUTO) factorizations
+def test_pointer_array_variants_match_strided(kl, ku):
+    n, nrhs, batch = 50, 2, 9
     A = I.gen_band(n, n, kl, ku, count=batch)
     B = I.gen_rhs(n, nrhs, count=batch)
     Ao, Bo = A.copy(), B.copy()
@@ -555,7 +556,7 @@ def test_fused_gbsv_kernel_vs_oracle_and_two_launch_plan(kl, ku, n):
     assert plan["fused"] and plan["kernels"][0] in ("gbtrf_rows_kernel", "gbtrf_cols_kernel")
     assert bl.trfs_plan(n, kl, ku, 1, batch, bl.TRFS_FUSED)["kernels"] == ["gbtrf_rows_kernel"]
     two = bl.trfs_plan(n, kl, ku, 1, batch, bl.TRFS_TWO_LAUNCH)["kernels"][0]
-    assert two == "gbtrf_rows_kernel"  # one right-hand side: the row-slot forward-fused factorization
+    assert two == ("gbtrf_cols_kernel" if bl.cols_available(kl, ku) else "gbtrf_rows_kernel")
     A = I.gen_band(n, n, kl, ku, count=batch, first=n)
     B = I.gen_rhs(n, 1, ldb=n + 2, count=batch, first=n)
     Ao, Bo = A.copy(), B.copy()
@@ -718,8 +719,8 @@ def test_cols_kernel_parity(kl, ku, n):
 @pytest.mark.parametrize("n,batch", [(5, 9), (40, 33), (257, 70)])
 @pytest.mark.parametrize("nrhs", [1, 3, 4, 16])
 def test_cols_trfs_forward_parity(kl, ku, n, batch, nrhs):
-    # nrhs > 1: the column-owner factorization with the forward substitution of all right-hand
-    # sides, then the backward solve; nrhs = 1: the row-slot / window plan (parity either way)
+    # the column-owner factorization with the forward substitution of all right-hand sides, then
+    # the backward solve
     """dgbtrfs on a column-owner band (factorization with the forward substitution on the fly,
     then the backward solve): factors, pivots and solution bitwise vs oracle dgbtrf + dgbtrs."""
     if not bl.cols_available(kl, ku):
@@ -733,8 +734,7 @@ def test_cols_trfs_forward_parity(kl, ku, n, batch, nrhs):
     oracle.dgbtrs(Ao, ipo, Bo, n, kl, ku)
     plan = bl.trfs_plan(n, kl, ku, nrhs, batch, bl.TRFS_TWO_LAUNCH)
     assert plan["bytes"] == ["trf_fwd", "trs_bwd"], plan
-    if nrhs > 1:  # the right-hand sides ride with the column-owner factorization
-        assert plan["kernels"][0] == "gbtrf_cols_kernel", plan
+    assert plan["kernels"][0] == "gbtrf_cols_kernel", plan  # the right-hand sides ride with it
     Ag, Bg = torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda()
     Pg = torch.zeros((batch, n), dtype=torch.int32, device="cuda")
     Ig = torch.full((batch,), -7, dtype=torch.int32, device="cuda")
