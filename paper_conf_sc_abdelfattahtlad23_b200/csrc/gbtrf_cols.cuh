@@ -48,13 +48,16 @@ struct TrfCols {
     static constexpr int WARPS = 4;
     static constexpr size_t smem_bytes() { return (size_t)WARPS * GPW * GROUP_DBL * sizeof(double); }
     static constexpr int MINB_SMEM = (int)((227 * 1024) / smem_bytes());
-    // resident CTAs per SM: 4 (128 registers); 2 (255 registers) for windows of >= 9 doubles per
-    // lane -- (2,32) with 16 lanes x 3 slots measured 2.03 ms at 128 registers, 1.42 ms at 255 (C4)
+    // resident CTAs per SM (C4's (2,32), 16 lanes x 3 slots, measured): the factorization alone 3
+    // (168 registers: 1.28 ms vs 1.47 at 255 and 2.03 at 128); with the 16 right-hand sides 2
+    // (255 registers: 1.78 ms vs 1.94 at 168); 4 (128 registers) for the small windows
 #ifndef BANDLU_COLS_MINB
-#define BANDLU_COLS_MINB (CPL * (KL + 1) >= 9 ? 2 : 4)
+#define BANDLU_COLS_MINB(fwd) (CPL * (KL + 1) >= 9 ? ((fwd) && GL >= 16 ? 2 : 3) : 4)
 #endif
-    static constexpr int MINB =
-        MINB_SMEM < BANDLU_COLS_MINB ? (MINB_SMEM < 1 ? 1 : MINB_SMEM) : BANDLU_COLS_MINB;
+    static constexpr int minb(bool fwd) {
+        return MINB_SMEM < BANDLU_COLS_MINB(fwd) ? (MINB_SMEM < 1 ? 1 : MINB_SMEM) : BANDLU_COLS_MINB(fwd);
+    }
+    static constexpr int MINB = minb(false);
 };
 
 // |x| as a 64-bit integer key from the two words (integer ops only; the 64-bit
@@ -65,7 +68,7 @@ __device__ __forceinline__ uint64_t abs_key_w(double x) {
 }
 
 template <int KL, int KU, int GL, int CPL, int FL, class AP, class PP, class BP>
-__global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<KL, KU, GL, CPL>::MINB)
+__global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<KL, KU, GL, CPL>::minb((FL & 1) != 0))
     gbtrf_cols_kernel(int n, AP A, int ldab, PP P, int *__restrict__ info, int batch, BP Bv, int nrhs, int ldb) {
     using C = TrfCols<KL, KU, GL, CPL>;
     constexpr bool FWD = FL & 1, BWD = FL & 2;  // FL_FWD, FL_BWD (gbtrf_rows.cuh)
