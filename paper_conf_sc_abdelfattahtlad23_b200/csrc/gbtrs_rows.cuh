@@ -41,7 +41,10 @@ struct TrsRows {
     static constexpr int KL = KL_, KU = KU_, KV = KL + KU;
     static constexpr int G = pow2_ceil(KV + 1 > 2 ? KV + 1 : 2);  // lanes per matrix
     static constexpr int GPW = 32 / G;                           // matrices per warp
-    static constexpr int P = 8;                                  // factor prefetch distance (steps)
+#ifndef BANDLU_TRS_ROWS_P
+#define BANDLU_TRS_ROWS_P 8
+#endif
+    static constexpr int P = BANDLU_TRS_ROWS_P;                  // factor prefetch distance (steps)
     static constexpr int WARPS = 4;                              // warps per CTA
     static_assert(KV + 1 <= 32, "one lane per window row");
 };
