@@ -48,7 +48,13 @@ __global__ void __launch_bounds__(32) gbtrs_bwd_kernel(int n, AP A, int ldab, BP
     constexpr int gpw = GPW;  // matrices per warp
     extern __shared__ __align__(16) double smem[];
     const int lane = (int)lane_id();
+    // [r2b] (-DBANDLU_BWD_REVERSE_ORDER) warps taking the batch from its end, where the preceding
+    // factorization's last columns may still sit in L2, measured slower: C3 0.290 vs 0.286 ms
+#ifdef BANDLU_BWD_REVERSE_ORDER
+    const int64_t base = (int64_t)(gridDim.x - 1 - blockIdx.x) * gpw;
+#else
     const int64_t base = (int64_t)blockIdx.x * gpw;
+#endif
 
     // ---- copy role: lane -> (matrix cm of the warp, chunk phase cq)
     constexpr int CPG = 32 / GPW;
