@@ -26,6 +26,13 @@
 //    active window.
 // Interchanges are relabelings (reading 10), IAMAX is first-max
 // (exact 64-bit key compare, ties by smallest logical row; reading 2).
+//
+// Build-time experiment flags (DESIGN.md Sec. 6 records each measurement; none is on by default):
+//   exact variants  BANDLU_ROWS_FASTCHAIN, _SHFL_P, _LOOKAHEAD, _REC64, _KEY64, _NOHOIST, _LDS64,
+//                   _IPIV_STEP, _Y_BLOCK, _NBLK, _U, _MAXREG, _MINW -- bitwise equal, measured
+//                   slower or equal;
+//   timing-only     BANDLU_ABL_NOSTAGE, _NOOUT, _NOREC, _NOSHIFT, _NOSEARCH, _NORCP, _HALF --
+//                   remove work to see what it costs; their RESULTS ARE WRONG (never in the library).
 #pragma once
 #include "backsolve_fused.cuh"
 #include "common.cuh"
