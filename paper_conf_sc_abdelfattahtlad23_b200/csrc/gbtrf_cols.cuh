@@ -204,9 +204,21 @@ __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<
 
 #pragma unroll 1
     for (int j0 = 0; j0 < n; j0 += GL) {
+        // [r2b] the GL steps of a ring turn run as GL/UB passes of an UB-step unrolled body: only the
+        // step's position in its staging block (o) indexes registers; the owner lane (s) is a
+        // run-time value (C4, GL = 16: code 4x smaller -- the instruction-cache misses were 12.6% of
+        // the stall samples -- and 120-136 instead of 168-210 registers)
+#ifdef BANDLU_COLS_FULL_UNROLL
+#define BANDLU_COLS_SB_STEP GL
+#else
+#define BANDLU_COLS_SB_STEP UB
+#endif
+#pragma unroll 1
+        for (int sb = 0; sb < GL && j0 + sb < n; sb += BANDLU_COLS_SB_STEP) {
 #pragma unroll
-        for (int s = 0; s < GL; ++s) {
-            const int j = j0 + s, o = s % UB, b = j / UB;
+        for (int so_ = 0; so_ < BANDLU_COLS_SB_STEP; ++so_) {
+            const int s = sb + so_;
+            const int j = j0 + s, o = so_ % UB, b = j / UB;
             if (j >= n) break;
             if (o == 0) stage_block(b + 2);
             // ---- row j+KL enters as position KL (zero outside its band / beyond n)
@@ -336,10 +348,12 @@ __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<
                     cp_async_wait<1>();
                     __syncwarp();
                 }
-                if (s + 1 < GL) fetch_incoming(j + 1, s + 1, j0);
-                else fetch_incoming(j + 1, 0, j0 + GL);  // the next ring turn (slots rotate below)
+                const bool turn = (s + 1 == GL);  // the next ring turn (slots rotate below)
+                fetch_incoming(j + 1, turn ? 0 : s + 1, turn ? j0 + GL : j0);
             }
         }
+        }
+#undef BANDLU_COLS_SB_STEP
         // ---- ring turn: slot k <- slot k+1, the retired slot 0 (columns j0+NR+t) goes last
 #pragma unroll
         for (int r = 0; r <= KL; ++r) {
