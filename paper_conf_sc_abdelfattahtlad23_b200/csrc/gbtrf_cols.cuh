@@ -44,18 +44,20 @@ struct TrfCols {
     static constexpr int BIT = (BK * UB + GL - 1) / GL;
     // per group: NSB staging blocks + one output block (UB x BKP each) + NSB x UB x GL entries of
     // the right-hand sides (FL_FWD: lane t carries right-hand side t, nrhs <= GL)
-    static constexpr int GROUP_DBL = (NSB + 1) * UB * BKP + NSB * UB * GL;
+    // (the right-hand-side staging only with FL_FWD)
+    __host__ __device__ static constexpr int group_dbl(bool fwd) { return (NSB + 1) * UB * BKP + (fwd ? NSB * UB * GL : 0); }
+    static constexpr int GROUP_DBL = group_dbl(true);
     static constexpr int WARPS = 4;
-    static constexpr size_t smem_bytes() { return (size_t)WARPS * GPW * GROUP_DBL * sizeof(double); }
-    static constexpr int MINB_SMEM = (int)((227 * 1024) / smem_bytes());
-    // resident CTAs per SM (C4's (2,32), 16 lanes x 3 slots, measured): the factorization alone 3
-    // (168 registers: 1.28 ms vs 1.47 at 255 and 2.03 at 128); with the 16 right-hand sides 2
-    // (255 registers: 1.78 ms vs 1.94 at 168); 4 (128 registers) for the small windows
+    static constexpr size_t smem_bytes(bool fwd = true) { return (size_t)WARPS * GPW * group_dbl(fwd) * sizeof(double); }
+    static constexpr int minb_smem(bool fwd) { return (int)((227 * 1024) / smem_bytes(fwd)); }
+    // resident CTAs per SM, shared memory permitting: 4 (128 registers) for the small windows;
+    // C4's (2,32) (16 lanes x 3 slots, 120-136 registers since the UB-step passes) measured best at
+    // 3 for the factorization alone (1.10 ms; 1.18 at 4) and 2-3 with the 16 right-hand sides
 #ifndef BANDLU_COLS_MINB
 #define BANDLU_COLS_MINB(fwd) (CPL * (KL + 1) >= 9 ? ((fwd) && GL >= 16 ? 2 : 3) : 4)
 #endif
     static constexpr int minb(bool fwd) {
-        return MINB_SMEM < BANDLU_COLS_MINB(fwd) ? (MINB_SMEM < 1 ? 1 : MINB_SMEM) : BANDLU_COLS_MINB(fwd);
+        return minb_smem(true) < BANDLU_COLS_MINB(fwd) ? (minb_smem(true) < 1 ? 1 : minb_smem(true)) : BANDLU_COLS_MINB(fwd);
     }
     static constexpr int MINB = minb(false);
 };
@@ -143,7 +145,10 @@ __global__ void __launch_bounds__(TrfCols<KL, KU, GL, CPL>::WARPS * 32, TrfCols<
             const int cc = cc0 + i * (GL / UB);
             if (i * (GL / UB) < BK) {
                 const bool ok = rowok && cc < BK && (cc - so >= 0) && (cc - so <= KV) && (j0b + cc < nl);
-                const double x = ld_shared_f64(src0 + (uint32_t)(i * (GL / UB) * 8));
+                // (cc >= BK would read past the output block -- past the group's shared memory for
+                // the last group of a CTA: predicated off, like the store)
+                double x = 0.0;
+                ld_shared_f64_if(cc < BK, src0 + (uint32_t)(i * (GL / UB) * 8), x);
                 st_global_f64_if(ok, dst + i * xstride, x);
             }
         }
