@@ -98,6 +98,10 @@ namespace {
 
 // (KL, KU, GL, CPL) compiled as column-owner kernels (gbtrf_cols.cuh; kl <= 4, square): GL lanes
 // per matrix with CPL column slots each (GL*CPL >= kl+ku+1); AUTO's choice where compiled.
+#ifndef BANDLU_COLS_C4_GL  // (2,32): lanes per matrix x column slots per lane (experiments: 32 x 2)
+#define BANDLU_COLS_C4_GL 16
+#define BANDLU_COLS_C4_CPL 3
+#endif
 #if defined(BANDLU_NO_COLS)
 #define BANDLU_COLS_LIST(X)
 #elif defined(BANDLU_ONLY_C3)
@@ -111,7 +115,28 @@ namespace {
     X(2, 3, 4, 2)           \
     X(3, 0, 4, 1)           \
     X(3, 2, 4, 2)           \
-    X(2, 32, 16, 3)         \
+    X(2, 32, BANDLU_COLS_C4_GL, BANDLU_COLS_C4_CPL) \
+    BANDLU_COLS_EXTRA(X)
+#endif
+// the same bands with the forward substitution riding along (dgbtrfs): (2,32) with 32 lanes x 2
+// slots there (one lane per right-hand side up to 32; C4: 1.62 vs 1.73 ms for 16 x 3), while the
+// factorization alone runs 16 x 3 (1.10 vs 1.54 ms for 32 x 2)
+#ifndef BANDLU_COLS_C4F_GL
+#define BANDLU_COLS_C4F_GL 32
+#define BANDLU_COLS_C4F_CPL 2
+#endif
+#if defined(BANDLU_NO_COLS) || defined(BANDLU_ONLY_C3)
+#define BANDLU_COLS_FWD_LIST(X) BANDLU_COLS_LIST(X)
+#else
+#define BANDLU_COLS_FWD_LIST(X) \
+    X(0, 0, 4, 1)               \
+    X(0, 3, 4, 1)               \
+    X(1, 1, 4, 1)               \
+    X(2, 2, 4, 2)               \
+    X(2, 3, 4, 2)               \
+    X(3, 0, 4, 1)               \
+    X(3, 2, 4, 2)               \
+    X(2, 32, BANDLU_COLS_C4F_GL, BANDLU_COLS_C4F_CPL) \
     BANDLU_COLS_EXTRA(X)
 #endif
 // opt-in (measured): (4,4) slower than the row-slot kernel (XGC-like 0.096 vs
@@ -386,7 +411,7 @@ bool trf_cols_fused(int kl, int ku) {
 #ifdef BANDLU_COLS_FUSED
 #define X(a, b, g, c) \
     if (kl == a && ku == b) return FusedSolveAny<a + b, g>::ok;
-    BANDLU_COLS_LIST(X)
+    BANDLU_COLS_FWD_LIST(X)
 #undef X
 #endif
     (void)kl, (void)ku;
@@ -399,7 +424,7 @@ bool trf_cols_fused(int kl, int ku) {
 int trf_cols_rhs(int kl, int ku) {
 #define X(a, b, g, c) \
     if (kl == a && ku == b) return g;
-    BANDLU_COLS_LIST(X)
+    BANDLU_COLS_FWD_LIST(X)
 #undef X
     return 0;
 }
@@ -1034,7 +1059,7 @@ int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ld
         if constexpr (FusedSolveAny<a + b, g>::ok)                                                                \
             return launch_trf_cols<a, b, g, c, FL_FWD | FL_BWD>(n, A, ldab, P, info, batch, st, B, nrhs, ldb);   \
     }
-        BANDLU_COLS_LIST(X)
+        BANDLU_COLS_FWD_LIST(X)
 #undef X
         return BANDLU_ERR_UNSUPPORTED;
     }
@@ -1066,7 +1091,7 @@ int run_trfs(int n, int kl, int ku, int nrhs, AP A, int ldab, PP P, BP B, int ld
             r = nrhs == 1 ? launch_trs_bwd<a, b>(n, Ac, ldab, Pc, B, ldb, batch, st)                        \
                           : launch_trs_window<a, b>(n, nrhs, Ac, ldab, Pc, B, ldb, nullptr, batch, st, 0);  \
     }
-        BANDLU_COLS_LIST(X)
+        BANDLU_COLS_FWD_LIST(X)
 #undef X
         return r;
     }

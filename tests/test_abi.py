@@ -168,7 +168,7 @@ def test_trfs_plan_reports_the_launches(lib):
     p = b.trfs_plan(1024, 2, 32, 16, 5000)
     # C4: the 16 right-hand sides ride with the column-owner factorization, then the backward solve
     assert p["kernels"] == ["gbtrf_cols_kernel", "gbtrs_window_kernel"] and p["bytes"] == ["trf_fwd", "trs_bwd"]
-    p = b.trfs_plan(1024, 2, 32, 17, 5000)  # more right-hand sides than lanes: trf + trs
+    p = b.trfs_plan(1024, 2, 32, 33, 5000)  # more right-hand sides than lanes (32): trf + trs
     assert p["kernels"] == ["gbtrf_cols_kernel", "gbtrs_window_kernel"] and p["bytes"] == ["trf", "trs"]
     p = b.trfs_plan(100, 5, 9, 1, 10, b.TRFS_TWO_LAUNCH)  # (5,9): not instantiated ahead of time
     if b.jit_band(5, 9):  # run-time compiled (NVRTC) kernels
